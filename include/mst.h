@@ -1,0 +1,168 @@
+/*
+ * include/mst.h — C ABI of the B200 Boruvka minimum-spanning-forest hot path (libmst.so).
+ *
+ * Operation (§5, "Boruvka's Minimum Spanning Tree Algorithm"): given an
+ * edge-weighted undirected graph, repeatedly (1) find the minimum edge of each node whose
+ * other endpoint is in another component, (2) isolate the minimum inter-component edge of
+ * each component, (3) break the cycles of chosen edges at the component with minimum id,
+ * (4) merge every cycle/tree into its representative — "the process repeats until there is
+ * a single component. The inter-component minimum-weight edges are the MST" (L227).
+ * Realised as SURVEY.md §8(a) rows A0-A11; the per-row design is in DESIGN.md.
+ *
+ * Readings of the paper adopted by this ABI:
+ *   R1  ties between equal weights are broken by edge id: e < f <=> (w_e, e) <_lex (w_f, f);
+ *       the result is therefore the UNIQUE minimum spanning forest F* (bit-checkable);
+ *   R3  disconnected inputs give a spanning FOREST, |F*| = n - c (c = #connected comps);
+ *   R4  self-loops are legal input and never selected (L217 assumes none);
+ *   R5  parallel edges are legal and compete by (w, id);
+ *   R6  weights are uint32 (0 allowed); the total weight is an exact uint64.
+ *
+ * Conventions shared by every entry point
+ *   - Edge id e in [0, m) is the position in the caller's src/dst/w arrays.
+ *   - 0 <= n <= 2^31-1 and 0 <= m <= 2^31-1 (edge ids and 2m arcs fit in 32 bits).
+ *   - Every endpoint must satisfy 0 <= src[e], dst[e] < n, else MST_EINVAL (checked on the
+ *     device during the build, before anything else runs).
+ *   - No C++ exception crosses the ABI. All functions are thread-compatible per handle
+ *     (one thread at a time per handle; different handles are independent).
+ *   - On any non-OK status a message is available from mst_last_error() (thread-local).
+ *   - There is no CPU fallback: without a usable CUDA device every call that needs one
+ *     returns MST_ECUDA.
+ */
+#ifndef MST_H_
+#define MST_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st* mst_stream_t; /* == cudaStream_t; NULL = legacy default stream */
+
+typedef enum {
+    MST_OK = 0,
+    MST_EINVAL = 1,    /* bad argument: null pointer with m > 0, n/m out of range, endpoint >= n */
+    MST_ENOMEM = 2,    /* device allocation failed (nothing leaked)                           */
+    MST_ECUDA = 3,     /* CUDA runtime/launch error; handle may only be destroyed afterwards   */
+    MST_ENCCL = 4,     /* NCCL error in a distributed handle                                   */
+    MST_EINTERNAL = 5, /* an internal invariant failed (e.g. forest size != n - c)             */
+    MST_ENOTSUP = 6    /* feature not built into this library                                  */
+} mst_status;
+
+typedef struct mst_graph mst_graph; /* opaque; owned by the library */
+
+/* ------------------------------------------------------------------ build (row A0)
+ * mst_create — validate the COO input and build the device-resident arc arrays.
+ *   n, m     : vertex and edge counts (see conventions).
+ *   src, dst : DEVICE pointers, int32[m], caller-owned, read only during the call.
+ *   w        : DEVICE pointer, uint32[m], caller-owned, read only during the call.
+ *   out      : receives the handle; *out = NULL on any error (nothing is leaked).
+ * Builds the CSR of PAPER.md §6 L229 ("store each edge twice, once for each direction"):
+ * 2 arcs per non-self-loop edge, grouped by source vertex, each carrying the packed key
+ * (uint64(w) << 32 | e). All per-round buffers are allocated here once, sized for the
+ * worst case (§7.1: MST pre-allocation, "the sum of the nodes in all
+ * components is constant"); mst_run allocates nothing. Synchronous. */
+mst_status mst_create(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
+                      const uint32_t* w, mst_graph** out);
+
+/* mst_create_host — as mst_create but src/dst/w are HOST pointers (pageable or pinned);
+ * the library copies them to the device (input transferred to the GPU). */
+mst_status mst_create_host(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
+                           const uint32_t* w, mst_graph** out);
+
+/* ------------------------------------------------------------------ run (rows A1-A11)
+ * mst_run — compute the minimum spanning forest F* of the handle's graph.
+ *   stream          : all device work is enqueued on this stream (torch's current stream
+ *                     when called from the Python binding).
+ *   out_edge_ids    : DEVICE pointer, int32, caller-owned, capacity >= max(n-1, 0);
+ *                     receives the ids of F* in ASCENDING order.
+ *   out_num_edges   : HOST pointer; receives |F*| = n - c.
+ *   out_total_weight: HOST pointer; receives sum of w[e] over F* (exact uint64).
+ * Blocks until results are valid (per-round sizes come back to the host, §7.1
+ * L263 "kernel computes the future size and the host reads it"). Re-runnable: the arcs of
+ * the build are never overwritten, so the same handle gives the same output every call.
+ * After an error the handle may only be destroyed. */
+mst_status mst_run(mst_graph* g, mst_stream_t stream, int32_t* out_edge_ids,
+                   int64_t* out_num_edges, uint64_t* out_total_weight);
+
+/* mst_run_host — as mst_run but out_edge_ids is a HOST pointer (capacity >= max(n-1,0));
+ * the device->host copy of the ids is part of the call. */
+mst_status mst_run_host(mst_graph* g, mst_stream_t stream, int32_t* out_edge_ids_host,
+                        int64_t* out_num_edges, uint64_t* out_total_weight);
+
+/* mst_solve_host — one end-to-end call from host arrays to host results:
+ * mst_create_host + mst_run_host + mst_destroy. Device memory comes from a stream-ordered
+ * pool that the library keeps between calls, so repeated solves do not pay cudaMalloc. */
+mst_status mst_solve_host(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
+                          const uint32_t* w, int32_t* out_edge_ids_host,
+                          int64_t* out_num_edges, uint64_t* out_total_weight);
+
+/* mst_destroy — NULL-safe; frees every library allocation of the handle. */
+void mst_destroy(mst_graph* g);
+
+/* thread-local message describing the last non-OK status returned on this thread */
+const char* mst_last_error(void);
+
+/* ------------------------------------------------------------------ introspection
+ * Per-run statistics of the last mst_run on the handle. Sizes let the caller compute the
+ * algorithmic byte model of SURVEY.md §8(d); kernel times are filled only while profiling
+ * is enabled (CUDA events recorded on the run's stream around every launch). */
+#define MST_MAX_ROUNDS 64
+enum {
+    MST_K_INIT = 0,    /* A1 run init (best = inf, msf bits = 0, counters)            */
+    MST_K_MIN0 = 1,    /* A2 round-0 segmented min                                    */
+    MST_K_HOOK = 2,    /* A4 hook + A6 renumber scan                                  */
+    MST_K_JUMP = 3,    /* A5 pointer-jump + A6 map compose                            */
+    MST_K_FILTER = 4,  /* A8 fused relabel + filter + compaction + next-round min     */
+    MST_K_OUTPUT = 5,  /* A11 output compaction                                       */
+    MST_K_COMM = 6,    /* A3 cross-GPU MIN (distributed handles)                      */
+    MST_K_COUNT = 7
+};
+typedef struct {
+    int64_t n, m, arcs0;                  /* vertices, edges, A_0 = 2 * #non-loop edges  */
+    int32_t rounds;                       /* R: rounds executed by the last run          */
+    int32_t nranks, rank;                 /* 1/0 for single-GPU handles                  */
+    int64_t local_arcs0;                  /* arcs owned by this rank                     */
+    int64_t n_r[MST_MAX_ROUNDS];          /* live components entering round r            */
+    int64_t a_r[MST_MAX_ROUNDS];          /* alive (local) arcs entering round r         */
+    int64_t num_edges;                    /* |F*| of the last run                        */
+    uint64_t total_weight;
+    double build_ms;                      /* wall time of the build in mst_create*       */
+    int32_t profiling;                    /* 1 if the kernel timers below are valid      */
+    double kernel_ms[MST_K_COUNT];        /* summed event time per kernel kind           */
+    int64_t kernel_launches[MST_K_COUNT];
+    double round_filter_ms[MST_MAX_ROUNDS]; /* A2 (r=0 slot of kernel_ms) / A8 per round */
+    int64_t gpu_launches;                 /* kernels launched by the last run            */
+} mst_stats;
+
+mst_status mst_get_stats(const mst_graph* g, mst_stats* out);
+
+/* enable (1) / disable (0) per-launch CUDA-event timing for subsequent runs */
+mst_status mst_set_profiling(mst_graph* g, int enable);
+
+/* ------------------------------------------------------------------ multi-GPU (§8(e))
+ * One process per GPU (torchrun). Every rank passes the identical full input; rank g keeps
+ * the arcs whose source lies in its vertex range (ranges chosen from the CSR row offsets so
+ * that arcs are balanced). Each round ends with an NCCL allreduce-MIN of the component-best
+ * array over NVLink; hook/jump/renumber then run replicated, so every rank holds identical
+ * labels and returns the identical full forest. The paper is single-GPU;
+ * this exchange step is the north star's extension. */
+mst_status mst_get_unique_id(uint8_t id[128]); /* wraps ncclGetUniqueId (rank 0 calls) */
+mst_status mst_create_dist(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
+                           const uint32_t* w, const uint8_t id[128], int rank, int nranks,
+                           mst_graph** out);
+
+/* mst_create_sim — test aid: a single-GPU handle that splits the arcs into `nshards`
+ * source ranges exactly as mst_create_dist would for nranks = nshards, runs every shard's
+ * per-round work itself and combines the shard minima with a device MIN in place of the
+ * NCCL allreduce. Exercises the sharding/replication logic without a second GPU. */
+mst_status mst_create_sim(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
+                          const uint32_t* w, int nshards, mst_graph** out);
+
+/* library version string, e.g. "mst-b200 0.1 sm_100a" */
+const char* mst_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MST_H_ */
