@@ -1,0 +1,351 @@
+#!/usr/bin/env python
+"""Benchmark: MST edges/s of the B200 Boruvka hot path (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload rmat22] [--impl reference]
+
+One step = one ``mst_run`` (every round of A1-A11) over the workload's graph, which is
+built once (``mst_create``, reported separately as ``build_ms``) and resident in HBM.
+value = m * K / (sum of the K device-timed steps) — m = undirected input edges (reading R7).
+For N > 1 (torchrun) the edges are sharded by source range and every round ends with an
+NCCL allreduce-MIN; all ranks process the one graph: "strong" scaling,
+time = max over ranks. Rank 0 prints one JSON line.
+
+``--impl reference`` times the oracle (CPU Kruskal, test infrastructure) on the host cores
+on the same workload instead (this tier's reference arm).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "MST edges/sec (device-timed) at 1/2/4/8 B200; % HBM roofline per round"
+UNIT = "edges/s"
+DEFAULT_WORKLOAD = "rmat22"  # BASELINE.json north-star target: RMAT-22 on 1 GPU (configs[3])
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+# --------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi sampled every 200 ms during the timed region (B200_PROFILING.md)."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index=0):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1])); smax.append(float(f[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None,
+                "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# --------------------------------------------------------------------------- workloads
+def make_workload(name, seed=0):
+    import graphgen
+    t = time.perf_counter()
+    g = graphgen.config(name, s=seed)
+    return g, time.perf_counter() - t
+
+
+def cpu_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count()
+
+
+def cpu_model():
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True).stdout
+        for ln in out.splitlines():
+            if ln.startswith("Model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def time_oracle(g, budget_s=30.0):
+    """The oracle as it stands, 1 host thread. Full workload when it fits the budget."""
+    import oracle
+    ids, total, secs = oracle.kruskal(g.n, g.src, g.dst, g.w, with_time=True)
+    return ids, total, secs
+
+
+# --------------------------------------------------------------------------- GPU arm
+def byte_model(st):
+    """Algorithmic bytes."""
+    a = st["a_r"]
+    R = st["rounds"]
+    a_next = a[1:] + [0] if R else []
+    per_round = []
+    for r in range(R):
+        per_round.append({"filter_bytes": 16 * a[r] + 16 * (a_next[r] if r + 1 < R else 0)})
+    return per_round
+
+
+def run_gpu(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ppopp_nasrebp13_b200 as mstb
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.gpus > 1 and world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} needs torchrun with {args.gpus} ranks (WORLD_SIZE={world})")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    mstb.load()
+    g, gen_s = make_workload(args.workload, args.seed)
+    n, m = g.n, g.m
+    dsrc = torch.from_numpy(g.src).cuda()
+    ddst = torch.from_numpy(g.dst).cuda()
+    dw = torch.from_numpy(g.w.view(np.int32)).cuda()
+    if world > 1:
+        uid = torch.zeros(128, dtype=torch.uint8, device="cuda")
+        if rank == 0:
+            uid.copy_(torch.frombuffer(bytearray(mstb.mst_get_unique_id()), dtype=torch.uint8))
+        dist.broadcast(uid, 0)
+        h = mstb.MSTGraph(n, dsrc, ddst, dw, dist=(bytes(uid.cpu().numpy()), rank, world))
+    else:
+        h = mstb.MSTGraph(n, dsrc, ddst, dw)
+    del dsrc, ddst, dw
+    build_ms = h.stats()["build_ms"]
+    out_ids = torch.empty(max(n - 1, 1), dtype=torch.int32, device="cuda")
+    stream = torch.cuda.current_stream()
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")  # > 126 MB L2
+
+    for _ in range(args.warmup):
+        h.run(out_ids)
+    h.set_profiling(True)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    clocks = ClockSampler(local)
+    clocks.start()
+    step_ms, filt_ms, filt_bytes, filt_launches, launches = [], 0.0, 0, 0, 0
+    round_acc = None
+    barrier()
+    for _ in range(args.steps):
+        flush.zero_()                       # L2 flushed between timed steps (not timed)
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        ids, cnt, tot = h.run(out_ids)
+        e1.record(stream)
+        e1.synchronize()
+        step_ms.append(e0.elapsed_time(e1))
+        st = h.stats()
+        launches += st["gpu_launches"]
+        filt_ms += st["kernel_ms"]["filter"]
+        filt_launches += st["kernel_launches"]["filter"]
+        bm = byte_model(st)
+        filt_bytes += sum(x["filter_bytes"] for x in bm)
+        if round_acc is None:
+            round_acc = [{"r": r, "n_r": st["n_r"][r], "A_r": st["a_r"][r], "filter_ms": 0.0,
+                          "filter_bytes": bm[r]["filter_bytes"]} for r in range(st["rounds"])]
+        for r in range(st["rounds"]):
+            round_acc[r]["filter_ms"] += st["round_filter_ms"][r] / args.steps
+    barrier()
+    clk = clocks.stop()
+    total_ms = float(np.sum(step_ms))
+    if world > 1:
+        t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+    ids_np = ids.cpu().numpy()
+    st = h.stats()
+    peak, peak_src = measured_peaks()
+
+    # ---- e2e: host arrays in, host ids out, through the C ABI (mst_solve_host)
+    e2e = None
+    if world == 1 and args.e2e_steps > 0:
+        import torch as _t
+        pin = lambda a: _t.from_numpy(a).pin_memory().numpy()  # noqa: E731
+        hs, hd, hw = pin(g.src), pin(g.dst), pin(g.w.view(np.int32)).view(np.uint32)
+        hout = _t.empty(max(n - 1, 1), dtype=_t.int32).pin_memory().numpy()
+        mstb.mst_solve_host(n, hs, hd, hw, hout)  # warm the pool
+        ts = []
+        for _ in range(args.e2e_steps):
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            _, c2, t2 = mstb.mst_solve_host(n, hs, hd, hw, hout)
+            ts.append(time.perf_counter() - t0)
+            assert c2 == cnt and t2 == tot
+        e2e = {"value": m * len(ts) / float(np.sum(ts)), "unit": UNIT,
+               "h2d_bytes_per_step": 12 * m, "d2h_bytes_per_step": 4 * cnt + 16,
+               "steps": len(ts), "api": "mst_solve_host (create_host + run_host + destroy)"}
+
+    result = None
+    if rank == 0:
+        cpu = None
+        parity = "not checked"
+        if not args.no_oracle:
+            o_ids, o_tot, o_secs = time_oracle(g)
+            parity = "bit-exact" if (np.array_equal(ids_np, o_ids) and tot == o_tot) else "MISMATCH"
+            cpu = {"value": m / o_secs, "unit": UNIT, "cores": 1, "kind": "oracle",
+                   "sample": f"full workload ({m} edges), 1 run, 1 of {cpu_cores()} host cores "
+                             f"({cpu_model()}); timer covers key build + sort + union-find + id sort",
+                   "seconds": o_secs}
+        achieved = filt_bytes / (filt_ms * 1e-3) / 1e9 if filt_ms > 0 else None
+        traffic = None
+        tp = os.path.join(ROOT, "profiles", f"ncu_traffic_{args.workload}.json")
+        if os.path.exists(tp):
+            traffic = json.load(open(tp)).get("filter_dram_bytes_per_launch")
+        rounds = []
+        for rr in round_acc or []:
+            gbs = rr["filter_bytes"] / (rr["filter_ms"] * 1e-3) / 1e9 if rr["filter_ms"] > 0 else None
+            rounds.append({**rr, "filter_GBps": gbs, "frac": gbs / peak if gbs else None})
+        result = {
+            "metric": METRIC, "value": m * args.steps / (total_ms * 1e-3), "unit": UNIT,
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+            "config": {"workload": g.name, "n": n, "m": m, "arcs0": st["arcs0"],
+                       "rounds": st["rounds"], "seed": args.seed,
+                       "generator": "graphgen (SURVEY.md §8(d) recipe)",
+                       "l2": "flushed between timed steps (256 MB write); arcs > L2",
+                       "parallelism": f"edge-sharded x{world}" if world > 1 else "1 GPU",
+                       "build_ms": build_ms, "gen_s": gen_s},
+            "parity": parity,
+            "num_edges": cnt, "total_weight": tot,
+            "roofline": {"bound": "hbm", "kernel": "k_filter_min (A8)",
+                         "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak if achieved else None, "traffic": traffic,
+                         "peak_source": peak_src,
+                         "avg_launch_ms": filt_ms / max(filt_launches, 1),
+                         "bytes_per_launch": filt_bytes / max(filt_launches, 1),
+                         "share_of_step": filt_ms / total_ms if total_ms else None},
+            "rounds": rounds,
+            "kernel_ms_per_step": {k: v for k, v in st["kernel_ms"].items()},
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches,
+            "clocks": clk,
+        }
+    h.close()
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return result
+
+
+# --------------------------------------------------------------------------- reference arm
+def run_reference(args):
+    """The oracle as it stands (CPU Kruskal, 1 host thread) on the same workload."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return None
+    import oracle
+    g, _ = make_workload(args.workload, args.seed)
+    budget = args.ref_budget_s
+    # a bounded sample: the full graph when K+W runs fit the budget, else an edge prefix
+    _, _, t_full = oracle.kruskal(g.n, g.src, g.dst, g.w, with_time=True)
+    steps_total = args.steps + max(args.warmup - 1, 0)
+    m_s = g.m
+    if t_full * steps_total > budget:
+        m_s = max(1, int(g.m * budget / (t_full * steps_total)))
+    src, dst, w = g.src[:m_s], g.dst[:m_s], g.w[:m_s]
+    for _ in range(max(args.warmup - 1, 0)):
+        oracle.kruskal(g.n, src, dst, w, with_time=True)
+    secs = []
+    for _ in range(args.steps):
+        secs.append(oracle.kruskal(g.n, src, dst, w, with_time=True)[2])
+    tot = float(np.sum(secs))
+    val = m_s * args.steps / tot
+    sample = (f"{'full workload' if m_s == g.m else 'edge-id prefix'} ({m_s} of {g.m} edges) "
+              f"per step; 1 of {cpu_cores()} host cores ({cpu_model()})")
+    return {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": 0, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": tot * 1e3 / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "u64", "data": "synthetic", "impl": "reference",
+            "config": {"workload": g.name, "n": g.n, "m": g.m, "sample_m": m_s},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--workload", default=DEFAULT_WORKLOAD,
+                    choices=["grid64", "uniform", "road", "rmat22", "dense"])
+    ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-oracle", action="store_true")
+    ap.add_argument("--ref-budget-s", type=float, default=150.0)
+    args = ap.parse_args()
+    if args.warmup < 3 and args.impl == "ours":
+        print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)
+    res = run_reference(args) if args.impl == "reference" else run_gpu(args)
+    if res is not None:
+        print(json.dumps(res))
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,166 @@
+// common.cuh — device helpers shared by the MST kernels (sm_100a).
+//
+// Nothing here is MST arithmetic; it is the plumbing the kernels share: cache-hinted
+// loads/stores, warp segmented minimum, and the decoupled look-back tile-status protocol
+// used for every single-pass stream compaction / scan (rows A0, A4/A6, A8, A11 of
+// SURVEY.md §8(a); the paper's "explicit deletion" of PAPER.md §7.2 L273 done as a
+// single-pass scan instead of a global re-layout).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace mstk {
+
+typedef uint32_t u32;
+typedef uint64_t u64;
+
+constexpr u64 KEY_INF = ~0ull;          // "no edge" (SURVEY.md §8 notation: ∞ = UINT64_MAX)
+constexpr u32 FULL = 0xffffffffu;
+
+// ------------------------------------------------------------------ memory access
+// L2 eviction-priority policies (createpolicy): the arc streams are read once and marked
+// evict-first so the small, hot label maps (evict-last) stay resident in the 126 MB L2.
+__device__ __forceinline__ u64 pol_evict_first() {
+    u64 p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ u64 pol_evict_last() {
+    u64 p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+// Streamed once: no L1 allocation, L2 evict-first.
+__device__ __forceinline__ u32 ld_stream_u32(const u32* p, u64 pol) {
+    u32 v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;"
+                 : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ u64 ld_stream_u64(const u64* p, u64 pol) {
+    u64 v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u64 %0, [%1], %2;"
+                 : "=l"(v) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ void st_stream_u32(u32* p, u32 v, u64 pol) {
+    asm volatile("st.global.L1::no_allocate.L2::cache_hint.u32 [%0], %1, %2;"
+                 :: "l"(p), "r"(v), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void st_stream_u64(u64* p, u64 v, u64 pol) {
+    asm volatile("st.global.L1::no_allocate.L2::cache_hint.u64 [%0], %1, %2;"
+                 :: "l"(p), "l"(v), "l"(pol) : "memory");
+}
+// Gathers from the label maps: read-only in-kernel, keep in L2 (evict-last).
+__device__ __forceinline__ int ld_map(const int* p, u64 pol) {
+    int v;
+    asm volatile("ld.global.nc.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
+// Coherent (L2) read of a word other CTAs may be updating in this kernel.
+__device__ __forceinline__ u64 ld_relaxed_u64(const u64* p) {
+    u64 v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed_u64(u64* p, u64 v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ u32 ld_relaxed_u32(const u32* p) {
+    u32 v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed_u32(u32* p, u32 v) {
+    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+
+// Monotone minimum with a stale-read pre-check: values only ever decrease, so any earlier
+// (stale) value is >= the current one and a key that does not beat it cannot win; this
+// keeps losing candidates off the L2 atomic units. Returns true if the atomic was issued.
+__device__ __forceinline__ bool min_update(u64* p, u64 key) {
+    u64 cur = __ldcg(p);
+    if (key < cur) {
+        atomicMin(reinterpret_cast<unsigned long long*>(p), (unsigned long long)key);
+        return true;
+    }
+    return false;
+}
+
+__device__ __forceinline__ u32 lane_id() { return threadIdx.x & 31; }
+__device__ __forceinline__ u32 lanemask_lt() {
+    u32 r;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(r));
+    return r;
+}
+
+__device__ __forceinline__ u64 shfl_up_u64(u64 v, int off) {
+    return __shfl_up_sync(FULL, v, off);
+}
+
+// Inclusive segmented minimum over contiguous runs of a warp. `heads` is the ballot of
+// run-head flags (bit 0 must be set). After the call a run's TAIL lane holds the min over
+// its whole run; every lane holds the min over [its run head .. itself].
+__device__ __forceinline__ u64 warp_seg_min(u64 v, u32 heads, u32 lane) {
+    const u32 below = heads & (FULL >> (31 - lane));
+    const int head = 31 - __clz(below);
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+        u64 o = shfl_up_u64(v, off);
+        if ((int)lane - off >= head) v = o < v ? o : v;
+    }
+    return v;
+}
+
+// tails of contiguous runs given their heads: lane l is a tail iff l == 31 or l+1 is a head
+__device__ __forceinline__ u32 run_tails(u32 heads) { return (heads >> 1) | 0x80000000u; }
+
+// ------------------------------------------------------------------ decoupled look-back
+// Tile status word: [63:62] flag (0 = not ready, 1 = aggregate, 2 = inclusive prefix),
+// [61:32] epoch (30 bits, unique per launch so the status array is never cleared),
+// [31:0] value (counts < 2^32: arcs A_r <= 2m <= 2^32-2).
+constexpr u32 ST_AGG = 1, ST_PRE = 2;
+
+__device__ __forceinline__ u64 st_pack(u32 flag, u32 epoch, u32 value) {
+    return ((u64)flag << 62) | ((u64)(epoch & 0x3fffffffu) << 32) | (u64)value;
+}
+
+__device__ __forceinline__ void publish(u64* status, u32 tile, u32 flag, u32 epoch, u32 value) {
+    st_relaxed_u64(status + tile, st_pack(flag, epoch, value));
+}
+
+// Called by ONE full warp: returns the exclusive prefix of `tile` (sum of the values of all
+// tiles < tile). Deadlock-free when tiles are dispatched in increasing order (one CTA per
+// tile in blockIdx order, or a co-resident persistent grid walking tiles in order).
+__device__ __forceinline__ u32 lookback(const u64* status, u32 tile, u32 epoch) {
+    const u32 lane = lane_id();
+    const u32 ep = epoch & 0x3fffffffu;
+    u32 excl = 0;
+    long long base = (long long)tile - 32;
+    while (true) {
+        long long idx = base + lane;
+        u32 flag, val;
+        if (idx >= 0) {
+            u64 s;
+            do {
+                s = ld_relaxed_u64(status + idx);
+                flag = (u32)(s >> 62);
+                if ((u32)((s >> 32) & 0x3fffffffu) != ep) flag = 0;
+            } while (flag == 0);
+            val = (u32)s;
+        } else {
+            flag = ST_PRE;  // virtual tiles before 0: prefix 0
+            val = 0;
+        }
+        const u32 pmask = __ballot_sync(FULL, flag == ST_PRE);
+        if (pmask) {
+            const u32 hi = 31 - __clz(pmask);
+            excl += __reduce_add_sync(FULL, lane >= hi ? val : 0u);
+            return excl;
+        }
+        excl += __reduce_add_sync(FULL, val);
+        base -= 32;
+    }
+}
+
+}  // namespace mstk

@@ -1,0 +1,656 @@
+// mst_api.cu — the C ABI (include/mst.h) and the round loop that drives the kernels.
+//
+// Round structure (§5 L227 and the host loop of Fig. 3,
+// "the process repeats until there is a single component"):
+//
+//   A1  init   best_0 = inf, forest bits = 0
+//   A2  min0   best_0[v] = min key over v's arcs                        [A3: MIN over ranks]
+//   loop r = 0, 1, ...
+//     A4/A6 hook   parent, forest edges, keep-scan -> new ids, n_{r+1}, best_{r+1} = inf
+//     A5/A6 jump   roots, M_r = new id of root (-1: finished)
+//     A8    filter relabel + delete intra-component arcs + dedup + compact + best_{r+1}
+//     host reads (n_{r+1}, A_{r+1})      (kernel computes sizes, host reads)
+//     A10   stop when n_{r+1} == 0, or (single GPU) A_{r+1} == 0       [A3 before the next]
+//   A11 output ascending ids, count, total weight
+//
+// Nothing is allocated inside mst_run (PAPER.md L259 pre-allocation). All work is enqueued
+// on the caller's stream.
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/mst.h"
+#include "kernels.h"
+
+using namespace mstk;
+
+namespace {
+
+thread_local std::string g_err;
+
+mst_status fail(mst_status s, const char* fmt, ...) {
+    char buf[1024];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return s;
+}
+
+#define CK(call)                                                                          \
+    do {                                                                                  \
+        cudaError_t e_ = (call);                                                          \
+        if (e_ != cudaSuccess) {                                                          \
+            return fail(e_ == cudaErrorMemoryAllocation ? MST_ENOMEM : MST_ECUDA,         \
+                        "%s: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__,        \
+                        __LINE__);                                                        \
+        }                                                                                 \
+    } while (0)
+
+#define CKN(call)                                                                         \
+    do {                                                                                  \
+        ncclResult_t r_ = (call);                                                         \
+        if (r_ != ncclSuccess)                                                            \
+            return fail(MST_ENCCL, "%s: %s (%s:%d)", #call, ncclGetErrorString(r_),        \
+                        __FILE__, __LINE__);                                              \
+    } while (0)
+
+#define CKS(call)                                                                         \
+    do {                                                                                  \
+        mst_status s_ = (call);                                                           \
+        if (s_ != MST_OK) return s_;                                                      \
+    } while (0)
+
+// device-counter slots
+enum { C_ERR = 0, C_OUT = 1, C_NNEXT = 2, C_ANEXT = 3 };
+
+struct Shard {
+    u64 lo, hi;  // arc range [lo, hi) in arcs_0 and in the ping-pong buffers
+    u32 A;       // alive arcs entering the current round
+};
+
+struct ProfRec {
+    int kind, round;
+    cudaEvent_t a, b;
+};
+
+}  // namespace
+
+struct mst_graph {
+    int dev = 0, nsm = 148;
+    int64_t n = 0, m = 0;
+    u64 A0 = 0, nwords = 0;
+    cudaStream_t cst = nullptr;  // internal stream (create / destroy)
+    std::vector<void*> allocs;
+
+    u32 *eu = nullptr, *ev = nullptr, *row = nullptr;
+    u32 *s0 = nullptr, *d0 = nullptr;
+    u64* k0 = nullptr;
+    u32 *sbuf[2] = {nullptr, nullptr}, *dbuf[2] = {nullptr, nullptr};
+    u64* kbuf[2] = {nullptr, nullptr};
+    u64 *bestA = nullptr, *bestB = nullptr, *shard_best = nullptr;
+    u32* P = nullptr;
+    int *Mtmp = nullptr, *maps = nullptr;
+    u32* msf = nullptr;
+    u64* status = nullptr;
+    u32 epoch = 1;
+    u32* dcnt = nullptr;
+    u64* acc = nullptr;
+    u32* hcnt = nullptr;  // pinned
+    u64* hacc = nullptr;  // pinned
+    int* out_tmp = nullptr;  // for mst_run_host
+
+    std::vector<Shard> shards;  // local shards (1, or G in the simulation)
+    bool sim = false;
+    int rank = 0, nranks = 1;
+    ncclComm_t comm = nullptr;
+    bool dedup = true;
+
+    bool prof = false;
+    std::vector<ProfRec> recs;
+    std::vector<cudaEvent_t> evpool;
+    size_t evused = 0;
+    mst_stats st{};
+    bool broken = false;
+};
+
+namespace {
+
+bool g_pool_configured = false;
+
+mst_status configure_pool(int dev) {
+    if (g_pool_configured) return MST_OK;
+    cudaMemPool_t pool;
+    CK(cudaDeviceGetDefaultMemPool(&pool, dev));
+    uint64_t thr = UINT64_MAX;
+    CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+    g_pool_configured = true;
+    return MST_OK;
+}
+
+template <typename T>
+mst_status galloc(mst_graph* g, T** p, u64 count) {
+    u64 bytes = std::max<u64>(count * sizeof(T), 16);
+    void* q = nullptr;
+    cudaError_t e = cudaMallocAsync(&q, bytes, g->cst);
+    if (e != cudaSuccess) {
+        (void)cudaGetLastError();
+        return fail(e == cudaErrorMemoryAllocation ? MST_ENOMEM : MST_ECUDA,
+                    "device allocation of %llu bytes failed: %s", (unsigned long long)bytes,
+                    cudaGetErrorString(e));
+    }
+    g->allocs.push_back(q);
+    *p = reinterpret_cast<T*>(q);
+    return MST_OK;
+}
+
+void release(mst_graph* g) {
+    if (!g) return;
+    if (g->comm) ncclCommDestroy(g->comm);
+    if (g->cst) {
+        for (void* p : g->allocs) cudaFreeAsync(p, g->cst);
+        cudaStreamSynchronize(g->cst);
+    }
+    if (g->hcnt) cudaFreeHost(g->hcnt);
+    if (g->hacc) cudaFreeHost(g->hacc);
+    for (auto e : g->evpool) cudaEventDestroy(e);
+    if (g->cst) cudaStreamDestroy(g->cst);
+    delete g;
+}
+
+// --------------------------------------------------------------------------- profiling
+cudaEvent_t next_event(mst_graph* g) {
+    if (g->evused == g->evpool.size()) {
+        cudaEvent_t e;
+        cudaEventCreate(&e);
+        g->evpool.push_back(e);
+    }
+    return g->evpool[g->evused++];
+}
+
+struct Prof {
+    mst_graph* g;
+    cudaStream_t s;
+    int kind, round;
+    cudaEvent_t a = nullptr;
+    Prof(mst_graph* g_, cudaStream_t s_, int kind_, int round_)
+        : g(g_), s(s_), kind(kind_), round(round_) {
+        if (g->prof) {
+            a = next_event(g);
+            cudaEventRecord(a, s);
+        }
+        g->st.gpu_launches++;
+    }
+    ~Prof() {
+        if (g->prof) {
+            cudaEvent_t b = next_event(g);
+            cudaEventRecord(b, s);
+            g->recs.push_back({kind, round, a, b});
+        }
+    }
+};
+
+// --------------------------------------------------------------------------- build (A0)
+mst_status check_args(int64_t n, int64_t m, const void* src, const void* dst, const void* w) {
+    if (n < 0 || n > INT32_MAX) return fail(MST_EINVAL, "n = %lld out of [0, 2^31-1]", (long long)n);
+    if (m < 0 || m > INT32_MAX) return fail(MST_EINVAL, "m = %lld out of [0, 2^31-1]", (long long)m);
+    if (m > 0 && (!src || !dst || !w)) return fail(MST_EINVAL, "null input pointer with m > 0");
+    if (m > 0 && n == 0) return fail(MST_EINVAL, "m > 0 edges on n = 0 vertices");
+    return MST_OK;
+}
+
+// Arc-balanced source ranges: shard g owns sources [v_g, v_{g+1}) with v_g the first vertex
+// whose row offset reaches g * A0 / G (computed from the CSR row offsets).
+mst_status shard_ranges(mst_graph* g, int G, std::vector<u64>& lo, std::vector<u64>& hi) {
+    lo.assign(G, 0);
+    hi.assign(G, 0);
+    if (G == 1) {
+        hi[0] = g->A0;
+        return MST_OK;
+    }
+    std::vector<u32> row(g->n + 1);
+    CK(cudaMemcpyAsync(row.data(), g->row, (g->n + 1) * sizeof(u32), cudaMemcpyDeviceToHost,
+                       g->cst));
+    CK(cudaStreamSynchronize(g->cst));
+    std::vector<u64> vb(G + 1);
+    vb[0] = 0;
+    vb[G] = g->n;
+    for (int j = 1; j < G; ++j) {
+        const u64 target = g->A0 * (u64)j / (u64)G;
+        vb[j] = (u64)(std::lower_bound(row.begin(), row.end(), (u32)target) - row.begin());
+        vb[j] = std::max(vb[j], vb[j - 1]);
+        vb[j] = std::min<u64>(vb[j], g->n);
+    }
+    for (int j = 0; j < G; ++j) {
+        lo[j] = row[vb[j]];
+        hi[j] = row[vb[j + 1]];
+    }
+    return MST_OK;
+}
+
+mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w, int nshards_sim,
+                 int rank, int nranks) {
+    auto t0 = std::chrono::steady_clock::now();
+    const u64 n = g->n, m = g->m;
+    g->nwords = (m + 31) / 32;
+    CKS(galloc(g, &g->eu, m));
+    CKS(galloc(g, &g->ev, m));
+    CKS(galloc(g, &g->row, n + 1));
+    u32* deg;
+    u32* cursor;
+    CKS(galloc(g, &deg, n));
+    CKS(galloc(g, &cursor, n));
+    CKS(galloc(g, &g->dcnt, 8 + 64));
+    CKS(galloc(g, &g->acc, 4));
+    const u64 nslots = status_slots_needed(n, 2 * m, g->nwords);
+    CKS(galloc(g, &g->status, nslots));
+    CK(cudaMemsetAsync(g->status, 0, nslots * sizeof(u64), g->cst));
+    CK(cudaMemsetAsync(deg, 0, std::max<u64>(n, 1) * sizeof(u32), g->cst));
+    CK(cudaMemsetAsync(g->dcnt, 0, 72 * sizeof(u32), g->cst));
+    CK(cudaMallocHost(&g->hcnt, 72 * sizeof(u32)));
+    CK(cudaMallocHost(&g->hacc, 4 * sizeof(u64)));
+
+    CK(launch_degree(g->cst, g->nsm, (u32)n, (u32)m, src, dst, g->eu, g->ev, deg, g->dcnt + C_ERR));
+    CK(cudaMemcpyAsync(g->hcnt, g->dcnt, sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
+    CK(cudaStreamSynchronize(g->cst));
+    if (g->hcnt[0]) return fail(MST_EINVAL, "an endpoint is outside [0, n) (n = %lld)", (long long)n);
+
+    if (n > 0) {
+        CK(launch_scan_rows(g->cst, (u32)n, deg, g->row, cursor, g->status, g->epoch++));
+    } else {
+        CK(cudaMemsetAsync(g->row, 0, sizeof(u32), g->cst));
+    }
+    u32 A0;
+    CK(cudaMemcpyAsync(&A0, g->row + n, sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
+    CK(cudaStreamSynchronize(g->cst));
+    g->A0 = A0;
+    CKS(galloc(g, &g->s0, A0));
+    CKS(galloc(g, &g->d0, A0));
+    CKS(galloc(g, &g->k0, A0));
+    CK(launch_scatter(g->cst, g->nsm, (u32)m, g->eu, g->ev, w, cursor, g->s0, g->d0, g->k0));
+
+    // shards: simulation = all G ranges locally; distributed = this rank's range only
+    const int G = nshards_sim > 1 ? nshards_sim : nranks;
+    std::vector<u64> lo, hi;
+    CKS(shard_ranges(g, G, lo, hi));
+    g->shards.clear();
+    u64 cap = 0;
+    for (int j = 0; j < G; ++j) {
+        if (nshards_sim <= 1 && j != rank) continue;
+        g->shards.push_back({lo[j], hi[j], (u32)(hi[j] - lo[j])});
+        cap = std::max(cap, hi[j]);
+    }
+    // ping-pong arc buffers: a shard's arcs keep their [lo, hi) window in every buffer
+    for (int b = 0; b < 2; ++b) {
+        CKS(galloc(g, &g->sbuf[b], cap));
+        CKS(galloc(g, &g->dbuf[b], cap));
+        CKS(galloc(g, &g->kbuf[b], cap));
+    }
+    CKS(galloc(g, &g->bestA, n));
+    CKS(galloc(g, &g->bestB, n));
+    if (g->sim) CKS(galloc(g, &g->shard_best, n * (u64)g->shards.size()));
+    CKS(galloc(g, &g->P, n));
+    CKS(galloc(g, &g->Mtmp, n));
+    CKS(galloc(g, &g->maps, 2 * n + 1));  // sum_r n_r <= 2n: every live component merges
+    CKS(galloc(g, &g->msf, g->nwords));
+    CK(cudaStreamSynchronize(g->cst));
+    g->st.n = g->n;
+    g->st.m = g->m;
+    g->st.arcs0 = (int64_t)g->A0;
+    g->st.nranks = nranks;
+    g->st.rank = rank;
+    u64 local = 0;
+    for (auto& s : g->shards) local += s.hi - s.lo;
+    g->st.local_arcs0 = (int64_t)local;
+    g->st.build_ms =
+        std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    return MST_OK;
+}
+
+mst_status create_common(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
+                         const uint32_t* w, int nshards_sim, const uint8_t* id, int rank,
+                         int nranks, mst_graph** out) {
+    if (!out) return fail(MST_EINVAL, "out is NULL");
+    *out = nullptr;
+    CKS(check_args(n, m, src, dst, w));
+    if (nranks < 1 || rank < 0 || rank >= nranks) return fail(MST_EINVAL, "bad rank/nranks");
+    if (nshards_sim < 1 || nshards_sim > 64) return fail(MST_EINVAL, "nshards must be in [1, 64]");
+    int dev;
+    CK(cudaGetDevice(&dev));
+    CKS(configure_pool(dev));
+    mst_graph* g = new (std::nothrow) mst_graph();
+    if (!g) return fail(MST_ENOMEM, "host allocation failed");
+    g->dev = dev;
+    g->n = n;
+    g->m = m;
+    g->sim = nshards_sim > 1;
+    g->rank = rank;
+    g->nranks = nranks;
+    if (const char* e = getenv("MST_DEDUP")) g->dedup = atoi(e) != 0;
+    cudaError_t e = cudaDeviceGetAttribute(&g->nsm, cudaDevAttrMultiProcessorCount, dev);
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&g->cst, cudaStreamNonBlocking);
+    if (e != cudaSuccess) {
+        release(g);
+        return fail(MST_ECUDA, "device setup: %s", cudaGetErrorString(e));
+    }
+    mst_status s = build(g, src, dst, (const unsigned*)w, nshards_sim, rank, nranks);
+    if (s == MST_OK && nranks > 1) {
+        ncclUniqueId uid;
+        memcpy(&uid, id, sizeof uid);
+        ncclResult_t r = ncclCommInitRank(&g->comm, nranks, uid, rank);
+        if (r != ncclSuccess) s = fail(MST_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
+    }
+    if (s != MST_OK) {
+        std::string keep = g_err;
+        (void)cudaGetLastError();
+        release(g);
+        g_err = keep;
+        return s;
+    }
+    *out = g;
+    return MST_OK;
+}
+
+// --------------------------------------------------------------------------- run
+mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out_num,
+                    uint64_t* out_total) {
+    const u64 n = g->n;
+    g->recs.clear();
+    g->evused = 0;
+    g->st.gpu_launches = 0;
+    g->st.rounds = 0;
+    for (int j = 0; j < MST_K_COUNT; ++j) {
+        g->st.kernel_ms[j] = 0;
+        g->st.kernel_launches[j] = 0;
+    }
+    for (int r = 0; r < MST_MAX_ROUNDS; ++r) {
+        g->st.n_r[r] = g->st.a_r[r] = 0;
+        g->st.round_filter_ms[r] = 0;
+    }
+    if (n == 0) {
+        *out_num = 0;
+        *out_total = 0;
+        g->st.num_edges = 0;
+        g->st.total_weight = 0;
+        return MST_OK;
+    }
+    const int G = (int)g->shards.size();
+    // ---- A1 init
+    {
+        Prof p(g, s, MST_K_INIT, 0);
+        CK(cudaMemsetAsync(g->bestA, 0xff, n * sizeof(u64), s));
+        CK(cudaMemsetAsync(g->msf, 0, std::max<u64>(g->nwords, 1) * sizeof(u32), s));
+        CK(cudaMemsetAsync(g->acc, 0, 4 * sizeof(u64), s));
+        if (g->sim) CK(cudaMemsetAsync(g->shard_best, 0xff, n * G * sizeof(u64), s));
+    }
+    // ---- A2 round-0 minimum (+ A3)
+    for (int j = 0; j < G; ++j) {
+        Shard& sh = g->shards[j];
+        sh.A = (u32)(sh.hi - sh.lo);
+        u64* tgt = g->sim ? g->shard_best + (u64)j * n : g->bestA;
+        if (sh.A == 0) continue;
+        Prof p(g, s, MST_K_MIN0, 0);
+        CK(launch_min0(s, sh.A, g->s0 + sh.lo, g->k0 + sh.lo, tgt));
+    }
+    if (g->sim) {
+        Prof p(g, s, MST_K_COMM, 0);
+        CK(launch_combine_min(s, g->nsm, (u32)n, G, g->shard_best, n, g->bestA));
+    } else if (g->comm) {
+        Prof p(g, s, MST_K_COMM, 0);
+        CKN(ncclAllReduce(g->bestA, g->bestA, n, ncclUint64, ncclMin, g->comm, s));
+    }
+
+    MapChain chain;
+    chain.len = 0;
+    u64 moff = 0;
+    u32 nr = (u32)n;
+    u64* bcur = g->bestA;
+    u64* bnxt = g->bestB;
+    int r = 0, outb = 0;
+    bool first = true;
+    while (true) {
+        if (r >= MST_MAX_ROUNDS || chain.len >= MST_CHAIN_MAX)
+            return fail(MST_EINTERNAL, "round limit exceeded (r = %d)", r);
+        u64 asum = 0;
+        for (auto& sh : g->shards) asum += sh.A;
+        g->st.n_r[r] = nr;
+        g->st.a_r[r] = (int64_t)asum;
+        int* Mr = g->maps + moff;
+        {
+            Prof p(g, s, MST_K_HOOK, r);
+            CK(launch_hook(s, nr, bcur, bnxt, g->eu, g->ev, chain, g->P, g->Mtmp, g->msf, g->acc,
+                           g->status, g->epoch++, g->dcnt + C_NNEXT));
+        }
+        {
+            Prof p(g, s, MST_K_JUMP, r);
+            CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, Mr));
+        }
+        for (int j = 0; j < G; ++j) {
+            Shard& sh = g->shards[j];
+            u64* tgt = g->sim ? g->shard_best + (u64)j * n : bnxt;
+            if (sh.A == 0) {
+                CK(cudaMemsetAsync(g->dcnt + C_ANEXT + j, 0, sizeof(u32), s));
+                continue;
+            }
+            const u32* si = first ? g->s0 + sh.lo : g->sbuf[outb ^ 1] + sh.lo;
+            const u32* di = first ? g->d0 + sh.lo : g->dbuf[outb ^ 1] + sh.lo;
+            const u64* ki = first ? g->k0 + sh.lo : g->kbuf[outb ^ 1] + sh.lo;
+            Prof p(g, s, MST_K_FILTER, r);
+            CK(launch_filter_min(s, g->dedup, sh.A, si, di, ki, Mr, g->sbuf[outb] + sh.lo,
+                                 g->dbuf[outb] + sh.lo, g->kbuf[outb] + sh.lo, tgt, g->status,
+                                 g->epoch++, g->dcnt + C_ANEXT + j));
+        }
+        CK(cudaMemcpyAsync(g->hcnt, g->dcnt, (C_ANEXT + G) * sizeof(u32), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        const u32 nn = g->hcnt[C_NNEXT];
+        u64 anext = 0;
+        for (int j = 0; j < G; ++j) {
+            g->shards[j].A = g->hcnt[C_ANEXT + j];
+            anext += g->shards[j].A;
+        }
+        chain.m[chain.len++] = Mr;
+        moff += nr;
+        ++r;
+        first = false;
+        outb ^= 1;
+        if (nn == 0) break;
+        if (!g->comm && anext == 0) break;
+        if (moff + nn > 2 * n + 1) return fail(MST_EINTERNAL, "label-map storage overflow");
+        if (g->sim) {
+            Prof p(g, s, MST_K_COMM, r);
+            CK(launch_combine_min(s, g->nsm, nn, G, g->shard_best, n, bnxt));
+        } else if (g->comm) {
+            Prof p(g, s, MST_K_COMM, r);
+            CKN(ncclAllReduce(bnxt, bnxt, nn, ncclUint64, ncclMin, g->comm, s));
+        }
+        std::swap(bcur, bnxt);
+        nr = nn;
+    }
+    g->st.rounds = r;
+    // ---- A11 output
+    {
+        Prof p(g, s, MST_K_OUTPUT, r);
+        if (g->nwords) {
+            CK(launch_output(s, (u32)g->nwords, g->msf, out_ids, g->status, g->epoch++,
+                             g->dcnt + C_OUT));
+        } else {
+            CK(cudaMemsetAsync(g->dcnt + C_OUT, 0, sizeof(u32), s));
+        }
+    }
+    CK(cudaMemcpyAsync(g->hcnt, g->dcnt, 2 * sizeof(u32), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(g->hacc, g->acc, 2 * sizeof(u64), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if ((u64)g->hcnt[C_OUT] != g->hacc[1])
+        return fail(MST_EINTERNAL, "forest size mismatch: %u ids vs %llu hooks", g->hcnt[C_OUT],
+                    (unsigned long long)g->hacc[1]);
+    if (g->hacc[1] >= n) return fail(MST_EINTERNAL, "forest has >= n edges");
+    *out_num = (int64_t)g->hacc[1];
+    *out_total = g->hacc[0];
+    g->st.num_edges = *out_num;
+    g->st.total_weight = *out_total;
+    if (g->prof) {
+        for (auto& rc : g->recs) {
+            float ms = 0;
+            cudaEventElapsedTime(&ms, rc.a, rc.b);
+            g->st.kernel_ms[rc.kind] += ms;
+            g->st.kernel_launches[rc.kind] += 1;
+            if (rc.kind == MST_K_FILTER && rc.round < MST_MAX_ROUNDS) g->st.round_filter_ms[rc.round] += ms;
+        }
+    }
+    g->st.profiling = g->prof ? 1 : 0;
+    return MST_OK;
+}
+
+template <typename F>
+mst_status guarded(F&& f) {
+    try {
+        return f();
+    } catch (const std::bad_alloc&) {
+        return fail(MST_ENOMEM, "host allocation failed");
+    } catch (...) {
+        return fail(MST_EINTERNAL, "unexpected C++ exception");
+    }
+}
+
+}  // namespace
+
+// =========================================================================== C ABI
+extern "C" {
+
+const char* mst_version(void) { return "mst-b200 0.1 sm_100a"; }
+
+const char* mst_last_error(void) { return g_err.c_str(); }
+
+mst_status mst_create(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
+                      const uint32_t* w, mst_graph** out) {
+    return guarded([&] { return create_common(n, m, src, dst, w, 1, nullptr, 0, 1, out); });
+}
+
+mst_status mst_create_sim(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
+                          const uint32_t* w, int nshards, mst_graph** out) {
+    return guarded([&] { return create_common(n, m, src, dst, w, nshards, nullptr, 0, 1, out); });
+}
+
+mst_status mst_get_unique_id(uint8_t id[128]) {
+    return guarded([&]() -> mst_status {
+        if (!id) return fail(MST_EINVAL, "id is NULL");
+        ncclUniqueId uid;
+        CKN(ncclGetUniqueId(&uid));
+        static_assert(sizeof(uid) == 128, "ncclUniqueId is 128 bytes");
+        memcpy(id, &uid, 128);
+        return MST_OK;
+    });
+}
+
+mst_status mst_create_dist(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
+                           const uint32_t* w, const uint8_t id[128], int rank, int nranks,
+                           mst_graph** out) {
+    return guarded([&]() -> mst_status {
+        if (nranks > 1 && !id) return fail(MST_EINVAL, "id is NULL");
+        return create_common(n, m, src, dst, w, 1, id, rank, nranks, out);
+    });
+}
+
+mst_status mst_create_host(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
+                           const uint32_t* w, mst_graph** out) {
+    return guarded([&]() -> mst_status {
+        if (!out) return fail(MST_EINVAL, "out is NULL");
+        *out = nullptr;
+        CKS(check_args(n, m, src, dst, w));
+        int dev;
+        CK(cudaGetDevice(&dev));
+        CKS(configure_pool(dev));
+        cudaStream_t st;
+        CK(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+        void *ds = nullptr, *dd = nullptr, *dw = nullptr;
+        const size_t b = std::max<size_t>((size_t)m * 4, 16);
+        cudaError_t e = cudaMallocAsync(&ds, b, st);
+        if (e == cudaSuccess) e = cudaMallocAsync(&dd, b, st);
+        if (e == cudaSuccess) e = cudaMallocAsync(&dw, b, st);
+        if (e == cudaSuccess && m > 0) e = cudaMemcpyAsync(ds, src, (size_t)m * 4, cudaMemcpyHostToDevice, st);
+        if (e == cudaSuccess && m > 0) e = cudaMemcpyAsync(dd, dst, (size_t)m * 4, cudaMemcpyHostToDevice, st);
+        if (e == cudaSuccess && m > 0) e = cudaMemcpyAsync(dw, w, (size_t)m * 4, cudaMemcpyHostToDevice, st);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+        mst_status s = MST_OK;
+        if (e != cudaSuccess)
+            s = fail(e == cudaErrorMemoryAllocation ? MST_ENOMEM : MST_ECUDA, "host->device input copy: %s",
+                     cudaGetErrorString(e));
+        else
+            s = create_common(n, m, (const int32_t*)ds, (const int32_t*)dd, (const uint32_t*)dw, 1,
+                              nullptr, 0, 1, out);
+        if (ds) cudaFreeAsync(ds, st);
+        if (dd) cudaFreeAsync(dd, st);
+        if (dw) cudaFreeAsync(dw, st);
+        cudaStreamSynchronize(st);
+        cudaStreamDestroy(st);
+        return s;
+    });
+}
+
+mst_status mst_run(mst_graph* g, mst_stream_t stream, int32_t* out_edge_ids,
+                   int64_t* out_num_edges, uint64_t* out_total_weight) {
+    return guarded([&]() -> mst_status {
+        if (!g) return fail(MST_EINVAL, "handle is NULL");
+        if (g->broken) return fail(MST_EINVAL, "handle is unusable after an earlier error");
+        if (!out_num_edges || !out_total_weight) return fail(MST_EINVAL, "null output pointer");
+        if (!out_edge_ids && g->n > 1) return fail(MST_EINVAL, "out_edge_ids is NULL");
+        mst_status s = run_impl(g, (cudaStream_t)stream, out_edge_ids, out_num_edges, out_total_weight);
+        if (s != MST_OK) g->broken = true;
+        return s;
+    });
+}
+
+mst_status mst_run_host(mst_graph* g, mst_stream_t stream, int32_t* out_ids_host,
+                        int64_t* out_num_edges, uint64_t* out_total_weight) {
+    return guarded([&]() -> mst_status {
+        if (!g) return fail(MST_EINVAL, "handle is NULL");
+        if (!out_ids_host && g->n > 1) return fail(MST_EINVAL, "out_edge_ids_host is NULL");
+        if (!g->out_tmp) CKS(galloc(g, &g->out_tmp, std::max<int64_t>(g->n - 1, 1)));
+        CK(cudaStreamSynchronize(g->cst));
+        CKS(mst_run(g, stream, g->out_tmp, out_num_edges, out_total_weight));
+        if (*out_num_edges > 0) {
+            CK(cudaMemcpyAsync(out_ids_host, g->out_tmp, (size_t)*out_num_edges * sizeof(int32_t),
+                               cudaMemcpyDeviceToHost, (cudaStream_t)stream));
+            CK(cudaStreamSynchronize((cudaStream_t)stream));
+        }
+        return MST_OK;
+    });
+}
+
+mst_status mst_solve_host(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
+                          const uint32_t* w, int32_t* out_ids_host, int64_t* out_num_edges,
+                          uint64_t* out_total_weight) {
+    mst_graph* g = nullptr;
+    mst_status s = mst_create_host(n, m, src, dst, w, &g);
+    if (s != MST_OK) return s;
+    s = mst_run_host(g, g->cst, out_ids_host, out_num_edges, out_total_weight);
+    std::string keep = g_err;
+    mst_destroy(g);
+    g_err = keep;
+    return s;
+}
+
+void mst_destroy(mst_graph* g) { release(g); }
+
+mst_status mst_get_stats(const mst_graph* g, mst_stats* out) {
+    if (!g || !out) return fail(MST_EINVAL, "null argument");
+    *out = g->st;
+    return MST_OK;
+}
+
+mst_status mst_set_profiling(mst_graph* g, int enable) {
+    if (!g) return fail(MST_EINVAL, "handle is NULL");
+    g->prof = enable != 0;
+    return MST_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,202 @@
+"""GPU parity: the CUDA path through the C ABI == the oracle, bit for bit (-m gpu).
+
+Compared on the same seeded inputs (graphgen): the ascending forest ids, their count and
+the exact uint64 total weight (integer work -> bit-exact, no tolerance).
+"""
+import numpy as np
+import pytest
+
+import mstcheck as mc
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def lib():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_ppopp_nasrebp13_b200 as p
+    p.load()
+    return p
+
+
+def dev(a, dt=torch.int32):
+    a = np.ascontiguousarray(a)
+    if a.dtype == np.uint32:
+        a = a.view(np.int32)
+    return torch.from_numpy(a.astype(np.int32, copy=False)).to("cuda")
+
+
+def gpu_msf(lib, n, src, dst, w, nshards=1, runs=1):
+    src = np.asarray(src, np.int32)
+    dst = np.asarray(dst, np.int32)
+    w = np.asarray(w, np.uint64).astype(np.uint32)
+    with lib.MSTGraph(n, dev(src), dev(dst), dev(w), nshards=nshards) as g:
+        outs = []
+        for _ in range(runs):
+            ids, cnt, tot = g.run()
+            outs.append((ids.cpu().numpy().copy(), cnt, tot))
+        st = g.stats()
+    for o in outs[1:]:  # re-runnable: same handle, same output
+        assert np.array_equal(o[0], outs[0][0]) and o[1:] == outs[0][1:]
+    return outs[0][0], outs[0][1], outs[0][2], st
+
+
+def assert_parity(lib, oracle_mod, n, src, dst, w, nshards=1, runs=1):
+    ids, cnt, tot, st = gpu_msf(lib, n, src, dst, w, nshards, runs)
+    o_ids, o_tot = oracle_mod.kruskal(n, src, dst, w)
+    assert cnt == len(o_ids), (cnt, len(o_ids))
+    assert tot == o_tot, (tot, o_tot)
+    assert np.array_equal(ids, o_ids)
+    return st
+
+
+# ------------------------------------------------------------------ fixtures and small graphs
+@pytest.mark.parametrize("name", ["hand_small.txt", "hand_forest.txt"])
+def test_golden(lib, oracle_mod, name):
+    import os
+    n, src, dst, w, exp = mc.load_golden(os.path.join(os.path.dirname(__file__), "golden", name))
+    ids, cnt, tot, _ = gpu_msf(lib, n, src, dst, w)
+    assert list(ids) == exp["expect_ids"] and tot == exp["expect_total"][0]
+
+
+def test_grid64(lib, oracle_mod, gg):
+    g = gg.config(1)
+    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, runs=3)
+    assert st["rounds"] >= 3
+
+
+@pytest.mark.parametrize("seed", range(120))
+def test_random_multigraphs(lib, oracle_mod, seed):
+    rng = np.random.default_rng(1000 + seed)
+    n = int(rng.integers(1, 10_000))
+    m = int(rng.integers(0, 6 * n))
+    wmax = [0, 1, 7, 1000, 2**32 - 1][seed % 5]
+    src, dst, w = mc.random_multigraph(rng, n, m, wmax)
+    assert_parity(lib, oracle_mod, n, src, dst, w)
+
+
+@pytest.mark.parametrize("seed", range(20))
+def test_tiny_graphs_vs_brute_force(lib, seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(1, 7)); m = int(rng.integers(0, 11))
+    src, dst, w = mc.random_multigraph(rng, n, m, 2)
+    ids, cnt, tot, _ = gpu_msf(lib, n, src, dst, w)
+    bf, bf_w, _ = mc.brute_force_msf(n, src, dst, w)
+    assert list(ids) == bf and tot == bf_w
+
+
+# ------------------------------------------------------------------ edge cases
+def test_empty_and_degenerate(lib, oracle_mod):
+    for n, src, dst, w in [(0, [], [], []), (1, [], [], []), (5, [], [], []),
+                           (3, [0, 1, 2], [0, 1, 2], [1, 2, 3]),   # self-loops only
+                           (2, [0], [1], [2**32 - 1]), (2, [1, 0, 1], [0, 1, 0], [3, 3, 3])]:
+        assert_parity(lib, oracle_mod, n, src, dst, w)
+
+
+def test_monotone_path_chain(lib, oracle_mod):
+    # every vertex hooks to its left neighbour in round 0: one chain of depth n-1
+    n = 1_000_000
+    src = np.arange(n - 1, dtype=np.int32)
+    st = assert_parity(lib, oracle_mod, n, src, src + 1, np.arange(1, n, dtype=np.uint32))
+    assert st["rounds"] <= 2
+
+
+def test_reverse_monotone_path_chain(lib, oracle_mod):
+    n = 300_000
+    src = np.arange(n - 1, dtype=np.int32)
+    assert_parity(lib, oracle_mod, n, src, src + 1, np.arange(n - 1, 0, -1).astype(np.uint32))
+
+
+def test_star_huge_degree(lib, oracle_mod):
+    # one segment spanning many CTAs (deg 10^6)
+    n = 1_000_001
+    rng = np.random.default_rng(3)
+    src = np.zeros(n - 1, np.int32)
+    dst = np.arange(1, n, dtype=np.int32)
+    w = rng.integers(0, 1000, n - 1).astype(np.uint32)
+    extra = rng.integers(1, n, 200_000).astype(np.int32)  # parallel + cross edges
+    src = np.concatenate([src, extra]); dst = np.concatenate([dst, np.roll(extra, 1)])
+    w = np.concatenate([w, rng.integers(0, 1000, 200_000).astype(np.uint32)])
+    assert_parity(lib, oracle_mod, n, src, dst, w)
+
+
+def test_all_equal_weights(lib, oracle_mod, gg):
+    g = gg.uniform(200_000, 800_000, 1, 2, 3, wlo=7, wmod=1)
+    assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w)
+
+
+def test_max_weights(lib, oracle_mod, gg):
+    g = gg.uniform(100_000, 300_000, 4, 5, 6, wlo=2**32 - 4, wmod=4)
+    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w)
+
+
+def test_many_components_and_isolated(lib, oracle_mod, gg):
+    g = gg.uniform(500_000, 200_000, 7, 8, 9)  # m < n: thousands of trees + isolated
+    assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w)
+
+
+def test_parallel_heavy(lib, oracle_mod, gg):
+    g = gg.uniform(64, 500_000, 11, 12, 13, wmod=50)
+    assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w)
+
+
+# ------------------------------------------------------------------ scaled configs
+@pytest.mark.parametrize("k,sd", [(2, 6), (3, 6), (4, 8), (5, 6), (2, 0)])
+def test_config_scaled(lib, oracle_mod, gg, k, sd):
+    g = gg.config(k, s=1, scale_down=sd)
+    assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, runs=2)
+
+
+@pytest.mark.parametrize("G", [2, 3, 8])
+@pytest.mark.parametrize("k,sd", [(1, 0), (4, 8), (3, 8)])
+def test_sim_shards(lib, oracle_mod, gg, G, k, sd):
+    g = gg.config(k, scale_down=sd)
+    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, nshards=G)
+    assert st["local_arcs0"] == st["arcs0"]
+
+
+# ------------------------------------------------------------------ API variants, errors
+def test_host_paths(lib, oracle_mod, gg):
+    g = gg.config(4, scale_down=8)
+    o_ids, o_tot = oracle_mod.kruskal(g.n, g.src, g.dst, g.w)
+    ids, cnt, tot = lib.mst_solve_host(g.n, g.src, g.dst, g.w)
+    assert np.array_equal(ids, o_ids) and tot == o_tot
+    with lib.MSTGraph(g.n, g.src, g.dst, g.w, host=True) as h:
+        ids, cnt, tot = h.run_host()
+        assert np.array_equal(ids, o_ids) and tot == o_tot
+
+
+def test_errors(lib):
+    with pytest.raises(lib.MSTError) as e:
+        lib.MSTGraph(3, dev([0, 1]), dev([1, 3]), dev([1, 1]))
+    assert e.value.status == 1
+    with pytest.raises(lib.MSTError) as e:
+        lib.MSTGraph(3, dev([0, -1]), dev([1, 2]), dev([1, 1]))
+    assert e.value.status == 1
+    with pytest.raises(lib.MSTError) as e:
+        lib.mst_solve_host(-1, np.array([], np.int32), np.array([], np.int32), np.array([], np.uint32))
+    assert e.value.status == 1
+    # a valid handle still works after failed creates (nothing leaked / poisoned)
+    ids, cnt, tot = lib.mst_solve_host(3, np.array([0, 1]), np.array([1, 2]), np.array([5, 6]))
+    assert list(ids) == [0, 1] and tot == 11
+
+
+def test_profiling_stats(lib, gg):
+    g = gg.config(2, scale_down=4)
+    with lib.MSTGraph(g.n, dev(g.src), dev(g.dst), dev(g.w)) as h:
+        h.set_profiling(True)
+        h.run()
+        st = h.stats()
+    assert st["profiling"] and st["kernel_ms"]["filter"] > 0
+    assert st["kernel_launches"]["filter"] == st["rounds"]
+    assert st["a_r"][0] == st["arcs0"] and st["n_r"][0] == g.n
+    assert all(a >= b for a, b in zip(st["n_r"], st["n_r"][1:]))
+
+
+# ------------------------------------------------------------------ full-size configs
+@pytest.mark.parametrize("k", [1, 2, 3, 4, 5])
+def test_full_size_configs(lib, oracle_mod, gg, k):
+    g = gg.config(k)
+    assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w)
