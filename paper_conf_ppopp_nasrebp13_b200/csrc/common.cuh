@@ -51,6 +51,17 @@ __device__ __forceinline__ void st_stream_u64(u64* p, u64 v, u64 pol) {
     asm volatile("st.global.L1::no_allocate.L2::cache_hint.u64 [%0], %1, %2;"
                  :: "l"(p), "l"(v), "l"(pol) : "memory");
 }
+// One arc record = 16 B {s, d, eid, w}: one LDG.128 / STG.128 per arc, coalesced.
+__device__ __forceinline__ uint4 ld_arc(const uint4* p, u64 pol) {
+    uint4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ void st_arc(uint4* p, uint4 v, u64 pol) {
+    asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.u32 [%0], {%1,%2,%3,%4}, %5;"
+                 :: "l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "l"(pol) : "memory");
+}
 // Gathers from the label maps: read-only in-kernel, keep in L2 (evict-last).
 __device__ __forceinline__ int ld_map(const int* p, u64 pol) {
     int v;
@@ -87,6 +98,15 @@ __device__ __forceinline__ bool min_update(u64* p, u64 key) {
     return false;
 }
 
+// Fire-and-forget minimum (RED, no return value, no pre-check load on the critical path).
+__device__ __forceinline__ void red_min_global(u64* p, u64 key) {
+    asm volatile("red.relaxed.gpu.global.min.u64 [%0], %1;" :: "l"(p), "l"(key) : "memory");
+}
+__device__ __forceinline__ void red_min_shared(u64* p, u64 key) {
+    asm volatile("red.shared.min.u64 [%0], %1;" :: "r"((u32)__cvta_generic_to_shared(p)), "l"(key)
+                 : "memory");
+}
+
 __device__ __forceinline__ u32 lane_id() { return threadIdx.x & 31; }
 __device__ __forceinline__ u32 lanemask_lt() {
     u32 r;
@@ -112,8 +132,99 @@ __device__ __forceinline__ u64 warp_seg_min(u64 v, u32 heads, u32 lane) {
     return v;
 }
 
+// Minimum key of my run of equal `s` among the 32 lanes (contiguous runs), computed with
+// two redux.sync over the run's lane mask: first the weight (hi word), then the edge id (lo
+// word) among the lanes holding that weight. Invalid lanes contribute (~0, ~0) = inf.
+// Returns the run min in (mh, ml) on every lane of the run and the run's first/last lane.
+__device__ __forceinline__ void run_min(u32 s, u32 hi, u32 lo, bool valid, u32 lane,
+                                        u32& mh, u32& ml, u32& head, u32& tail) {
+    const u32 ps = __shfl_up_sync(FULL, s, 1);
+    const u32 heads = __ballot_sync(FULL, lane == 0 || ps != s);
+    const u32 le = FULL >> (31 - lane);
+    head = 31 - __clz(heads & le);
+    const u32 above = heads & ~le;
+    tail = above ? (u32)(__ffs(above) - 2) : 31u;
+    const u32 mask = (FULL >> (31 - tail)) & (FULL << head);
+    const u32 v1 = valid ? hi : FULL;
+    mh = __reduce_min_sync(mask, v1);
+    const u32 v2 = (valid && hi == mh) ? lo : FULL;
+    ml = __reduce_min_sync(mask, v2);
+}
+
 // tails of contiguous runs given their heads: lane l is a tail iff l == 31 or l+1 is a head
 __device__ __forceinline__ u32 run_tails(u32 heads) { return (heads >> 1) | 0x80000000u; }
+
+// ------------------------------------------------------------------ TMA bulk copy + mbarrier
+// The producer warp streams arc tiles global -> shared with cp.async.bulk (SASS UBLKCP),
+// completion tracked by mbarrier transaction counts; consumers wait on the barrier's phase.
+__device__ __forceinline__ u32 smem_addr(const void* p) {
+    return (u32)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(u64* bar, u32 count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_addr(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(u64* bar, u32 bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;"
+                 :: "r"(smem_addr(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(u64* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_addr(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(u64* bar, u32 parity) {
+    const u32 a = smem_addr(bar);
+    asm volatile(
+        "{\n"
+        ".reg .pred P1;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+        "@!P1 bra WAIT_%=;\n"
+        "}\n" :: "r"(a), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, u32 bytes, u64* bar,
+                                            u64 pol) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+        " [%0], [%1], %2, [%3], %4;"
+        :: "r"(smem_addr(dst)), "l"(src), "r"(bytes), "r"(smem_addr(bar)), "l"(pol) : "memory");
+}
+// TMA bulk store shared -> global (survivor tiles); bulk-group completion tracking.
+__device__ __forceinline__ void tma_store_1d(void* dst, const void* src, u32 bytes, u64 pol) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;"
+                 :: "l"(dst), "r"(smem_addr(src)), "r"(bytes), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void bulk_commit() {
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_read0() {
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait0() {
+    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+}
+// generic-proxy shared-memory writes -> visible to the async proxy (TMA store)
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void named_arrive(u32 id, u32 nthreads) {
+    asm volatile("bar.arrive %0, %1;" :: "r"(id), "r"(nthreads) : "memory");
+}
+__device__ __forceinline__ void sts_arc(uint4* p, uint4 v) {
+    asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};"
+                 :: "r"(smem_addr(p)), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+}
+// named barrier among the consumer warps only (the producer warp never joins)
+__device__ __forceinline__ void named_sync(u32 id, u32 nthreads) {
+    asm volatile("bar.sync %0, %1;" :: "r"(id), "r"(nthreads) : "memory");
+}
+__device__ __forceinline__ uint4 lds_arc(const uint4* p) {
+    uint4 v;
+    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(smem_addr(p)));
+    return v;
+}
 
 // ------------------------------------------------------------------ decoupled look-back
 // Tile status word: [63:62] flag (0 = not ready, 1 = aggregate, 2 = inclusive prefix),

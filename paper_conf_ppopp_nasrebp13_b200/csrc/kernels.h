@@ -22,16 +22,16 @@ cudaError_t launch_degree(cudaStream_t st, int nsm, u32 n, u32 m, const int* src
 cudaError_t launch_scan_rows(cudaStream_t st, u32 n, const u32* deg, u32* row, u32* cursor,
                              u64* status, u32 epoch);
 cudaError_t launch_scatter(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
-                           const unsigned* w, u32* cursor, u32* s0, u32* d0, u64* k0);
-cudaError_t launch_min0(cudaStream_t st, u32 A, const u32* s, const u64* k, u64* best);
+                           const unsigned* w, u32* cursor, uint4* arcs);
+cudaError_t launch_min0(cudaStream_t st, int nsm, u64 A, const uint4* arcs, u64* best,
+                        u32* tile_ctrs, u32 seq);
 cudaError_t launch_hook(cudaStream_t st, u32 nr, const u64* best, u64* best_next, const u32* eu,
                         const u32* ev, const MapChain& chain, u32* P, int* Mtmp, u32* msf,
                         u64* acc, u64* status, u32 epoch, u32* n_next);
 cudaError_t launch_jump(cudaStream_t st, int nsm, u32 nr, u32* P, const int* Mtmp, int* Mr);
-cudaError_t launch_filter_min(cudaStream_t st, bool dedup, u32 A, const u32* s_in,
-                              const u32* d_in, const u64* k_in, const int* M, u32* s_out,
-                              u32* d_out, u64* k_out, u64* best, u64* status, u32 epoch,
-                              u32* a_next);
+cudaError_t launch_filter_min(cudaStream_t st, int nsm, u64 A, const uint4* in, const int* M,
+                              uint4* out, u64* best, const u32* nbest, u64* status, u32 epoch,
+                              u32* a_next, u32* tile_ctrs, u32 seq);
 cudaError_t launch_output(cudaStream_t st, u32 nwords, const u32* msf, int* out, u64* status,
                           u32 epoch, u32* out_count);
 cudaError_t launch_combine_min(cudaStream_t st, int nsm, u32 nr, int nshards, u64* shard_best,

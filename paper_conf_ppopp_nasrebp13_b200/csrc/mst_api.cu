@@ -71,7 +71,7 @@ mst_status fail(mst_status s, const char* fmt, ...) {
     } while (0)
 
 // device-counter slots
-enum { C_ERR = 0, C_OUT = 1, C_NNEXT = 2, C_ANEXT = 3 };
+enum { C_ERR = 0, C_OUT = 1, C_NNEXT = 2, C_TILE = 3, C_ANEXT = 5 };  // C_TILE: 2 slots
 
 struct Shard {
     u64 lo, hi;  // arc range [lo, hi) in arcs_0 and in the ping-pong buffers
@@ -93,16 +93,15 @@ struct mst_graph {
     std::vector<void*> allocs;
 
     u32 *eu = nullptr, *ev = nullptr, *row = nullptr;
-    u32 *s0 = nullptr, *d0 = nullptr;
-    u64* k0 = nullptr;
-    u32 *sbuf[2] = {nullptr, nullptr}, *dbuf[2] = {nullptr, nullptr};
-    u64* kbuf[2] = {nullptr, nullptr};
+    uint4* arcs0 = nullptr;                 // A_0 arcs {s, d, eid, w}, grouped by source
+    uint4* abuf[2] = {nullptr, nullptr};    // ping-pong alive arcs of rounds >= 1
     u64 *bestA = nullptr, *bestB = nullptr, *shard_best = nullptr;
     u32* P = nullptr;
     int *Mtmp = nullptr, *maps = nullptr;
     u32* msf = nullptr;
     u64* status = nullptr;
     u32 epoch = 1;
+    u32 pass_seq = 0;  // TMA arc-pass launches (tile-counter slot parity)
     u32* dcnt = nullptr;
     u64* acc = nullptr;
     u32* hcnt = nullptr;  // pinned
@@ -113,7 +112,6 @@ struct mst_graph {
     bool sim = false;
     int rank = 0, nranks = 1;
     ncclComm_t comm = nullptr;
-    bool dedup = true;
 
     bool prof = false;
     std::vector<ProfRec> recs;
@@ -273,10 +271,8 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CK(cudaMemcpyAsync(&A0, g->row + n, sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
     CK(cudaStreamSynchronize(g->cst));
     g->A0 = A0;
-    CKS(galloc(g, &g->s0, A0));
-    CKS(galloc(g, &g->d0, A0));
-    CKS(galloc(g, &g->k0, A0));
-    CK(launch_scatter(g->cst, g->nsm, (u32)m, g->eu, g->ev, w, cursor, g->s0, g->d0, g->k0));
+    CKS(galloc(g, &g->arcs0, A0));
+    CK(launch_scatter(g->cst, g->nsm, (u32)m, g->eu, g->ev, w, cursor, g->arcs0));
 
     // shards: simulation = all G ranges locally; distributed = this rank's range only
     const int G = nshards_sim > 1 ? nshards_sim : nranks;
@@ -290,11 +286,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
         cap = std::max(cap, hi[j]);
     }
     // ping-pong arc buffers: a shard's arcs keep their [lo, hi) window in every buffer
-    for (int b = 0; b < 2; ++b) {
-        CKS(galloc(g, &g->sbuf[b], cap));
-        CKS(galloc(g, &g->dbuf[b], cap));
-        CKS(galloc(g, &g->kbuf[b], cap));
-    }
+    for (int b = 0; b < 2; ++b) CKS(galloc(g, &g->abuf[b], cap));
     CKS(galloc(g, &g->bestA, n));
     CKS(galloc(g, &g->bestB, n));
     if (g->sim) CKS(galloc(g, &g->shard_best, n * (u64)g->shards.size()));
@@ -335,7 +327,6 @@ mst_status create_common(int64_t n, int64_t m, const int32_t* src, const int32_t
     g->sim = nshards_sim > 1;
     g->rank = rank;
     g->nranks = nranks;
-    if (const char* e = getenv("MST_DEDUP")) g->dedup = atoi(e) != 0;
     cudaError_t e = cudaDeviceGetAttribute(&g->nsm, cudaDevAttrMultiProcessorCount, dev);
     if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&g->cst, cudaStreamNonBlocking);
     if (e != cudaSuccess) {
@@ -399,7 +390,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         u64* tgt = g->sim ? g->shard_best + (u64)j * n : g->bestA;
         if (sh.A == 0) continue;
         Prof p(g, s, MST_K_MIN0, 0);
-        CK(launch_min0(s, sh.A, g->s0 + sh.lo, g->k0 + sh.lo, tgt));
+        CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, g->dcnt + C_TILE, g->pass_seq++));
     }
     if (g->sim) {
         Prof p(g, s, MST_K_COMM, 0);
@@ -441,13 +432,11 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                 CK(cudaMemsetAsync(g->dcnt + C_ANEXT + j, 0, sizeof(u32), s));
                 continue;
             }
-            const u32* si = first ? g->s0 + sh.lo : g->sbuf[outb ^ 1] + sh.lo;
-            const u32* di = first ? g->d0 + sh.lo : g->dbuf[outb ^ 1] + sh.lo;
-            const u64* ki = first ? g->k0 + sh.lo : g->kbuf[outb ^ 1] + sh.lo;
+            const uint4* in = (first ? g->arcs0 : g->abuf[outb ^ 1]) + sh.lo;
             Prof p(g, s, MST_K_FILTER, r);
-            CK(launch_filter_min(s, g->dedup, sh.A, si, di, ki, Mr, g->sbuf[outb] + sh.lo,
-                                 g->dbuf[outb] + sh.lo, g->kbuf[outb] + sh.lo, tgt, g->status,
-                                 g->epoch++, g->dcnt + C_ANEXT + j));
+            CK(launch_filter_min(s, g->nsm, sh.A, in, Mr, g->abuf[outb] + sh.lo, tgt,
+                                 g->dcnt + C_NNEXT, g->status, g->epoch++,
+                                 g->dcnt + C_ANEXT + j, g->dcnt + C_TILE, g->pass_seq++));
         }
         CK(cudaMemcpyAsync(g->hcnt, g->dcnt, (C_ANEXT + G) * sizeof(u32), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
