@@ -130,14 +130,21 @@ def time_oracle(g, budget_s=30.0):
 
 # --------------------------------------------------------------------------- GPU arm
 def byte_model(st):
-    """Algorithmic bytes."""
-    a = st["a_r"]
-    R = st["rounds"]
-    a_next = a[1:] + [0] if R else []
-    per_round = []
+    """Algorithmic bytes per round.
+
+    sparse round r (A8): 16 B read per alive arc + 16 B written per surviving arc; the round
+    that switches to the dense matrix writes no arcs (its minima go to the L2-resident
+    matrix). dense round r (A9): 8 B per matrix entry read (n_r (n_r - 1) / 2 entries)."""
+    a, R, dr = st["a_r"], st["rounds"], st.get("dense_round", -1)
+    out = []
     for r in range(R):
-        per_round.append({"filter_bytes": 16 * a[r] + 16 * (a_next[r] if r + 1 < R else 0)})
-    return per_round
+        dense = dr >= 0 and r >= dr
+        if dense:
+            out.append({"kind": "dense", "bytes": 8 * a[r]})
+        else:
+            nxt_sparse = r + 1 < R and not (dr >= 0 and r + 1 >= dr)
+            out.append({"kind": "filter", "bytes": 16 * a[r] + (16 * a[r + 1] if nxt_sparse else 0)})
+    return out
 
 
 def run_gpu(args):
@@ -202,10 +209,11 @@ def run_gpu(args):
         filt_ms += st["kernel_ms"]["filter"]
         filt_launches += st["kernel_launches"]["filter"]
         bm = byte_model(st)
-        filt_bytes += sum(x["filter_bytes"] for x in bm)
+        filt_bytes += sum(x["bytes"] for x in bm if x["kind"] == "filter")
         if round_acc is None:
-            round_acc = [{"r": r, "n_r": st["n_r"][r], "A_r": st["a_r"][r], "filter_ms": 0.0,
-                          "filter_bytes": bm[r]["filter_bytes"]} for r in range(st["rounds"])]
+            round_acc = [{"r": r, "kind": bm[r]["kind"], "n_r": st["n_r"][r], "A_r": st["a_r"][r],
+                          "filter_ms": 0.0, "filter_bytes": bm[r]["bytes"]}
+                         for r in range(st["rounds"])]
         for r in range(st["rounds"]):
             round_acc[r]["filter_ms"] += st["round_filter_ms"][r] / args.steps
     barrier()

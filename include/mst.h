@@ -116,7 +116,8 @@ enum {
     MST_K_FILTER = 4,  /* A8 fused relabel + filter + compaction + next-round min     */
     MST_K_OUTPUT = 5,  /* A11 output compaction                                       */
     MST_K_COMM = 6,    /* A3 cross-GPU MIN (distributed handles)                      */
-    MST_K_COUNT = 7
+    MST_K_DENSE = 7,   /* A9 dense rounds over the component min-matrix              */
+    MST_K_COUNT = 8
 };
 typedef struct {
     int64_t n, m, arcs0;                  /* vertices, edges, A_0 = 2 * #non-loop edges  */
@@ -131,8 +132,9 @@ typedef struct {
     int32_t profiling;                    /* 1 if the kernel timers below are valid      */
     double kernel_ms[MST_K_COUNT];        /* summed event time per kernel kind           */
     int64_t kernel_launches[MST_K_COUNT];
-    double round_filter_ms[MST_MAX_ROUNDS]; /* A2 (r=0 slot of kernel_ms) / A8 per round */
+    double round_filter_ms[MST_MAX_ROUNDS]; /* A8 (or A9 dense) kernel time per round     */
     int64_t gpu_launches;                 /* kernels launched by the last run            */
+    int32_t dense_round;                  /* first round run on the dense min-matrix, -1 */
 } mst_stats;
 
 mst_status mst_get_stats(const mst_graph* g, mst_stats* out);

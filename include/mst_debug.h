@@ -1,0 +1,26 @@
+/*
+ * include/mst_debug.h — test/benchmark-only entry points of libmst.so (not the product API).
+ *
+ * mst_debug_filter_pass: times the A8 kernel alone on the handle's
+ * round-0 arcs with a synthetic label map, so kernel variants can be measured in isolation:
+ *   map_kind 0: M[v] = v            (identity: every non-loop arc survives)
+ *   map_kind 1: M[v] = v / group    (contiguous blocks of `group` vertices per component)
+ *   map_kind 2: M[v] = h(v) % ncomp (hashed, ncomp = max(1, n / group) components)
+ *   stream     : device work is enqueued here; the call synchronises it.
+ *   iters      : timed repetitions (after one warm-up); *out_ms = mean ms per launch (CUDA
+ *                events on `stream`); *out_survivors = arcs kept by the last launch.
+ * The handle's per-round state is clobbered; run mst_run again before trusting it.
+ * Returns MST_EINVAL for bad arguments, MST_ECUDA on launch failure.
+ */
+#ifndef MST_DEBUG_H_
+#define MST_DEBUG_H_
+#include "mst.h"
+#ifdef __cplusplus
+extern "C" {
+#endif
+mst_status mst_debug_filter_pass(mst_graph* g, mst_stream_t stream, int map_kind, int64_t group,
+                                 int iters, double* out_ms, int64_t* out_survivors);
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -33,7 +33,7 @@ def sources():
 
 def deps():
     return sources() + glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(CSRC, "*.cuh")) + \
-        [os.path.join(ROOT, "include", "mst.h"), __file__]
+        glob.glob(os.path.join(ROOT, "include", "*.h")) + [__file__]
 
 
 def needs_build() -> bool:

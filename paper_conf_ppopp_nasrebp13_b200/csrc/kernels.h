@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 
 #define MST_CHAIN_MAX 64
+#define DENSE_MAX 4096  // components: the dense min-matrix then holds <= 8.4 M entries (67 MB)
 
 namespace mstk {
 typedef uint32_t u32;
@@ -31,10 +32,15 @@ cudaError_t launch_hook(cudaStream_t st, u32 nr, const u64* best, u64* best_next
 cudaError_t launch_jump(cudaStream_t st, int nsm, u32 nr, u32* P, const int* Mtmp, int* Mr);
 cudaError_t launch_filter_min(cudaStream_t st, int nsm, u64 A, const uint4* in, const int* M,
                               uint4* out, u64* best, const u32* nbest, u64* status, u32 epoch,
-                              u32* a_next, u32* tile_ctrs, u32 seq);
+                              u32* a_next, u32* tile_ctrs, u32 seq, u64* mat);
+cudaError_t launch_dense_init(cudaStream_t st, int nsm, const u32* n_ptr, u64* mat);
+cudaError_t launch_dense_round(cudaStream_t st, int nsm, u32 n, const u64* mat, const int* M,
+                               const u32* n_next, u64* mat_next, u64* best_next);
+u64 dense_entries(u64 n);
 cudaError_t launch_output(cudaStream_t st, u32 nwords, const u32* msf, int* out, u64* status,
                           u32 epoch, u32* out_count);
 cudaError_t launch_combine_min(cudaStream_t st, int nsm, u32 nr, int nshards, u64* shard_best,
                                u64 stride, u64* best);
 u64 status_slots_needed(u64 n, u64 arcs, u64 nwords);
+cudaError_t launch_debug_map(cudaStream_t st, u32 n, int kind, u32 group, int* M, u32* ncomp);
 }  // namespace mstk

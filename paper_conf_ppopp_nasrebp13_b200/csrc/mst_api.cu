@@ -28,6 +28,7 @@
 #include <vector>
 
 #include "../../include/mst.h"
+#include "../../include/mst_debug.h"
 #include "kernels.h"
 
 using namespace mstk;
@@ -99,6 +100,7 @@ struct mst_graph {
     u32* P = nullptr;
     int *Mtmp = nullptr, *maps = nullptr;
     u32* msf = nullptr;
+    u64* mat[2] = {nullptr, nullptr};  // dense min-matrices over component pairs
     u64* status = nullptr;
     u32 epoch = 1;
     u32 pass_seq = 0;  // TMA arc-pass launches (tile-counter slot parity)
@@ -294,6 +296,11 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CKS(galloc(g, &g->Mtmp, n));
     CKS(galloc(g, &g->maps, 2 * n + 1));  // sum_r n_r <= 2n: every live component merges
     CKS(galloc(g, &g->msf, g->nwords));
+    const char* dz = getenv("MST_DENSE");  // "0": keep every round sparse (tests, ablation)
+    if (n >= 2 && !(dz && dz[0] == '0')) {  // dense min-matrices (A9 / NEXT-1), <= 67 MB each
+        CKS(galloc(g, &g->mat[0], dense_entries(n)));
+        CKS(galloc(g, &g->mat[1], dense_entries(n)));
+    }
     CK(cudaStreamSynchronize(g->cst));
     g->st.n = g->n;
     g->st.m = g->m;
@@ -408,13 +415,16 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     u64* bnxt = g->bestB;
     int r = 0, outb = 0;
     bool first = true;
+    bool dense = false;  // this round's alive arcs live in the min-matrix g->mat[mc]
+    int mc = 0;
+    g->st.dense_round = -1;
     while (true) {
         if (r >= MST_MAX_ROUNDS || chain.len >= MST_CHAIN_MAX)
             return fail(MST_EINTERNAL, "round limit exceeded (r = %d)", r);
         u64 asum = 0;
         for (auto& sh : g->shards) asum += sh.A;
         g->st.n_r[r] = nr;
-        g->st.a_r[r] = (int64_t)asum;
+        g->st.a_r[r] = dense ? (int64_t)dense_entries(nr) : (int64_t)asum;
         int* Mr = g->maps + moff;
         {
             Prof p(g, s, MST_K_HOOK, r);
@@ -425,41 +435,64 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             Prof p(g, s, MST_K_JUMP, r);
             CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, Mr));
         }
-        for (int j = 0; j < G; ++j) {
-            Shard& sh = g->shards[j];
-            u64* tgt = g->sim ? g->shard_best + (u64)j * n : bnxt;
-            if (sh.A == 0) {
-                CK(cudaMemsetAsync(g->dcnt + C_ANEXT + j, 0, sizeof(u32), s));
-                continue;
+        if (dense) {
+            // A9/NEXT-1 dense round: scan the matrix, collapse into the next (smaller) one
+            Prof p(g, s, MST_K_DENSE, r);
+            CK(launch_dense_init(s, g->nsm, g->dcnt + C_NNEXT, g->mat[mc ^ 1]));
+            CK(launch_dense_round(s, g->nsm, nr, g->mat[mc], Mr, g->dcnt + C_NNEXT, g->mat[mc ^ 1],
+                                  bnxt));
+        } else {
+            if (g->mat[0]) CK(launch_dense_init(s, g->nsm, g->dcnt + C_NNEXT, g->mat[0]));
+            for (int j = 0; j < G; ++j) {
+                Shard& sh = g->shards[j];
+                u64* tgt = g->sim ? g->shard_best + (u64)j * n : bnxt;
+                if (sh.A == 0) {
+                    CK(cudaMemsetAsync(g->dcnt + C_ANEXT + j, 0, sizeof(u32), s));
+                    continue;
+                }
+                const uint4* in = (first ? g->arcs0 : g->abuf[outb ^ 1]) + sh.lo;
+                Prof p(g, s, MST_K_FILTER, r);
+                CK(launch_filter_min(s, g->nsm, sh.A, in, Mr, g->abuf[outb] + sh.lo, tgt,
+                                     g->dcnt + C_NNEXT, g->status, g->epoch++,
+                                     g->dcnt + C_ANEXT + j, g->dcnt + C_TILE, g->pass_seq++,
+                                     g->mat[0]));
             }
-            const uint4* in = (first ? g->arcs0 : g->abuf[outb ^ 1]) + sh.lo;
-            Prof p(g, s, MST_K_FILTER, r);
-            CK(launch_filter_min(s, g->nsm, sh.A, in, Mr, g->abuf[outb] + sh.lo, tgt,
-                                 g->dcnt + C_NNEXT, g->status, g->epoch++,
-                                 g->dcnt + C_ANEXT + j, g->dcnt + C_TILE, g->pass_seq++));
         }
         CK(cudaMemcpyAsync(g->hcnt, g->dcnt, (C_ANEXT + G) * sizeof(u32), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
         const u32 nn = g->hcnt[C_NNEXT];
         u64 anext = 0;
-        for (int j = 0; j < G; ++j) {
-            g->shards[j].A = g->hcnt[C_ANEXT + j];
-            anext += g->shards[j].A;
+        if (!dense) {
+            for (int j = 0; j < G; ++j) {
+                g->shards[j].A = g->hcnt[C_ANEXT + j];
+                anext += g->shards[j].A;
+            }
         }
+        const bool was_dense = dense;
         chain.m[chain.len++] = Mr;
         moff += nr;
         ++r;
         first = false;
         outb ^= 1;
-        if (nn == 0) break;
-        if (!g->comm && anext == 0) break;
+        if (nn <= 1) break;  // <= 1 live component: no inter-component edge is left
+        if (!dense && g->mat[0] && nn <= (u32)DENSE_MAX) {
+            dense = true;  // the filter just wrote the min-matrix g->mat[0]
+            mc = 0;
+            g->st.dense_round = r;
+        } else if (dense) {
+            mc ^= 1;
+        }
+        if (!dense && !g->comm && anext == 0) break;
         if (moff + nn > 2 * n + 1) return fail(MST_EINTERNAL, "label-map storage overflow");
-        if (g->sim) {
+        if (g->sim && !was_dense) {
             Prof p(g, s, MST_K_COMM, r);
             CK(launch_combine_min(s, g->nsm, nn, G, g->shard_best, n, bnxt));
-        } else if (g->comm) {
+        } else if (g->comm && !was_dense) {
             Prof p(g, s, MST_K_COMM, r);
             CKN(ncclAllReduce(bnxt, bnxt, nn, ncclUint64, ncclMin, g->comm, s));
+            if (dense)  // first dense round: every rank needs the full matrix
+                CKN(ncclAllReduce(g->mat[mc], g->mat[mc], dense_entries(nn), ncclUint64, ncclMin,
+                                  g->comm, s));
         }
         std::swap(bcur, bnxt);
         nr = nn;
@@ -492,7 +525,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             cudaEventElapsedTime(&ms, rc.a, rc.b);
             g->st.kernel_ms[rc.kind] += ms;
             g->st.kernel_launches[rc.kind] += 1;
-            if (rc.kind == MST_K_FILTER && rc.round < MST_MAX_ROUNDS) g->st.round_filter_ms[rc.round] += ms;
+            if ((rc.kind == MST_K_FILTER || rc.kind == MST_K_DENSE) && rc.round < MST_MAX_ROUNDS)
+                g->st.round_filter_ms[rc.round] += ms;
         }
     }
     g->st.profiling = g->prof ? 1 : 0;
@@ -640,6 +674,43 @@ mst_status mst_set_profiling(mst_graph* g, int enable) {
     if (!g) return fail(MST_EINVAL, "handle is NULL");
     g->prof = enable != 0;
     return MST_OK;
+}
+
+mst_status mst_debug_filter_pass(mst_graph* g, mst_stream_t stream, int map_kind, int64_t group,
+                                 int iters, double* out_ms, int64_t* out_survivors) {
+    return guarded([&]() -> mst_status {
+        if (!g || !out_ms || iters < 1 || g->n == 0 || g->shards.empty())
+            return fail(MST_EINVAL, "bad argument");
+        if (group < 1) group = 1;
+        cudaStream_t s = (cudaStream_t)stream;
+        const u64 n = g->n;
+        u32 ncomp = 0;
+        CK(launch_debug_map(s, (u32)n, map_kind, (u32)group, g->maps, &ncomp));
+        CK(cudaMemcpyAsync(g->dcnt + C_NNEXT, &ncomp, sizeof(u32), cudaMemcpyHostToDevice, s));
+        const Shard& sh = g->shards[0];
+        const u32 A = (u32)(sh.hi - sh.lo);
+        cudaEvent_t e0, e1;
+        CK(cudaEventCreate(&e0));
+        CK(cudaEventCreate(&e1));
+        for (int it = -1; it < iters; ++it) {
+            if (it == 0) CK(cudaEventRecord(e0, s));
+            CK(cudaMemsetAsync(g->bestB, 0xff, n * sizeof(u64), s));
+            CK(launch_filter_min(s, g->nsm, A, g->arcs0 + sh.lo, g->maps, g->abuf[0] + sh.lo,
+                                 g->bestB, g->dcnt + C_NNEXT, g->status, g->epoch++,
+                                 g->dcnt + C_ANEXT, g->dcnt + C_TILE, g->pass_seq++, nullptr));
+        }
+        CK(cudaEventRecord(e1, s));
+        CK(cudaEventSynchronize(e1));
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, e0, e1));
+        cudaEventDestroy(e0);
+        cudaEventDestroy(e1);
+        u32 surv = 0;
+        CK(cudaMemcpy(&surv, g->dcnt + C_ANEXT, sizeof(u32), cudaMemcpyDeviceToHost));
+        *out_ms = ms / iters;
+        if (out_survivors) *out_survivors = surv;
+        return MST_OK;
+    });
 }
 
 }  // extern "C"

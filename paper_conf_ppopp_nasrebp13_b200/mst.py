@@ -18,10 +18,11 @@ MST_OK, MST_EINVAL, MST_ENOMEM, MST_ECUDA, MST_ENCCL, MST_EINTERNAL, MST_ENOTSUP
 STATUS_NAMES = {0: "MST_OK", 1: "MST_EINVAL", 2: "MST_ENOMEM", 3: "MST_ECUDA", 4: "MST_ENCCL",
                 5: "MST_EINTERNAL", 6: "MST_ENOTSUP"}
 MAX_ROUNDS = 64
-K_INIT, K_MIN0, K_HOOK, K_JUMP, K_FILTER, K_OUTPUT, K_COMM, K_COUNT = range(8)
-KERNEL_NAMES = ["init", "min0", "hook", "jump", "filter", "output", "comm"]
+K_INIT, K_MIN0, K_HOOK, K_JUMP, K_FILTER, K_OUTPUT, K_COMM, K_DENSE, K_COUNT = range(9)
+KERNEL_NAMES = ["init", "min0", "hook", "jump", "filter", "output", "comm", "dense"]
 
 # every symbol include/mst.h declares
+DEBUG_EXPORTS = ["mst_debug_filter_pass"]  # include/mst_debug.h (test/bench only)
 EXPORTS = ["mst_create", "mst_create_host", "mst_run", "mst_run_host", "mst_solve_host",
            "mst_destroy", "mst_last_error", "mst_get_stats", "mst_set_profiling",
            "mst_get_unique_id", "mst_create_dist", "mst_create_sim", "mst_version"]
@@ -38,6 +39,7 @@ class mst_stats(ctypes.Structure):
         ("kernel_ms", ctypes.c_double * K_COUNT), ("kernel_launches", ctypes.c_int64 * K_COUNT),
         ("round_filter_ms", ctypes.c_double * MAX_ROUNDS),
         ("gpu_launches", ctypes.c_int64),
+        ("dense_round", ctypes.c_int32),
     ]
 
 
@@ -80,6 +82,9 @@ def load(build_if_missing: bool = True):
     L.mst_set_profiling.argtypes = [p, i32]
     L.mst_get_unique_id.argtypes = [p]
     L.mst_version.restype = ctypes.c_char_p
+    L.mst_debug_filter_pass.argtypes = [p, p, i32, i64, i32, ctypes.POINTER(ctypes.c_double),
+                                        ctypes.POINTER(ctypes.c_int64)]
+    L.mst_debug_filter_pass.restype = ctypes.c_int
     for name in EXPORTS:
         if name not in ("mst_destroy", "mst_last_error", "mst_version"):
             getattr(L, name).restype = ctypes.c_int
@@ -187,7 +192,16 @@ class MSTGraph:
             "kernel_launches": {KERNEL_NAMES[i]: s.kernel_launches[i] for i in range(K_COUNT)},
             "round_filter_ms": list(s.round_filter_ms[:R]),
             "gpu_launches": s.gpu_launches,
+            "dense_round": s.dense_round,
         }
+
+    def debug_filter_pass(self, map_kind=0, group=1, iters=5, stream=None):
+        """Times the A8 kernel alone on the round-0 arcs (include/mst_debug.h)."""
+        ms, surv = ctypes.c_double(0), ctypes.c_int64(0)
+        _check(load().mst_debug_filter_pass(self._h, _stream_ptr(stream), int(map_kind),
+                                            int(group), int(iters), ctypes.byref(ms),
+                                            ctypes.byref(surv)))
+        return ms.value, surv.value
 
     def close(self):
         if getattr(self, "_h", None):

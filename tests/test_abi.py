@@ -8,8 +8,8 @@ import pytest
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def header_symbols():
-    txt = open(os.path.join(ROOT, "include", "mst.h")).read()
+def header_symbols(name="mst.h"):
+    txt = open(os.path.join(ROOT, "include", name)).read()
     txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
     return sorted(set(re.findall(r"\b(mst_[a-z_]+)\s*\(", txt)))
 
@@ -17,12 +17,13 @@ def header_symbols():
 def test_header_symbols_listed_in_binding():
     import paper_conf_ppopp_nasrebp13_b200 as p
     assert header_symbols() == sorted(p.EXPORTS)
+    assert header_symbols("mst_debug.h") == sorted(p.mst.DEBUG_EXPORTS)
 
 
 def test_library_exports_every_declared_symbol():
     import paper_conf_ppopp_nasrebp13_b200 as p
     L = p.load()
-    for name in header_symbols():
+    for name in header_symbols() + header_symbols("mst_debug.h"):
         assert hasattr(L, name), name
     assert "sm_100a" in p.mst_version()
 

@@ -190,7 +190,8 @@ def test_profiling_stats(lib, gg):
         h.run()
         st = h.stats()
     assert st["profiling"] and st["kernel_ms"]["filter"] > 0
-    assert st["kernel_launches"]["filter"] == st["rounds"]
+    dr = st["dense_round"]
+    assert st["kernel_launches"]["filter"] == (dr if dr >= 0 else st["rounds"])
     assert st["a_r"][0] == st["arcs0"] and st["n_r"][0] == g.n
     assert all(a >= b for a, b in zip(st["n_r"], st["n_r"][1:]))
 
@@ -200,3 +201,20 @@ def test_profiling_stats(lib, gg):
 def test_full_size_configs(lib, oracle_mod, gg, k):
     g = gg.config(k)
     assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w)
+
+
+# ------------------------------------------------------------------ sparse-only rounds
+@pytest.mark.parametrize("k,sd", [(1, 0), (2, 6), (4, 8), (5, 6)])
+def test_sparse_only_rounds(lib, oracle_mod, gg, k, sd, monkeypatch):
+    """MST_DENSE=0 keeps every round on the compaction path (no dense min-matrix)."""
+    monkeypatch.setenv("MST_DENSE", "0")
+    g = gg.config(k, s=2, scale_down=sd)
+    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w)
+    assert st["dense_round"] == -1
+
+
+@pytest.mark.parametrize("k,sd", [(1, 0), (4, 6), (5, 6)])
+def test_dense_rounds_used(lib, oracle_mod, gg, k, sd):
+    g = gg.config(k, s=3, scale_down=sd)
+    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w)
+    assert st["dense_round"] >= 0
