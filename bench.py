@@ -134,15 +134,18 @@ def byte_model(st):
 
     sparse round r (A8): 16 B read per alive arc + 16 B written per surviving arc; the round
     that switches to the dense matrix writes no arcs (its minima go to the L2-resident
-    matrix). dense round r (A9): 8 B per matrix entry read (n_r (n_r - 1) / 2 entries)."""
+    matrix). dense round r (A9): 8 B per matrix entry read (n_r (n_r - 1) / 2 entries).
+    The last round only hooks (<= 1 live component is left) and moves no arcs."""
     a, R, dr = st["a_r"], st["rounds"], st.get("dense_round", -1)
     out = []
     for r in range(R):
         dense = dr >= 0 and r >= dr
-        if dense:
+        if r == R - 1:
+            out.append({"kind": "hook-only", "bytes": 0})
+        elif dense:
             out.append({"kind": "dense", "bytes": 8 * a[r]})
         else:
-            nxt_sparse = r + 1 < R and not (dr >= 0 and r + 1 >= dr)
+            nxt_sparse = not (dr >= 0 and r + 1 >= dr)
             out.append({"kind": "filter", "bytes": 16 * a[r] + (16 * a[r + 1] if nxt_sparse else 0)})
     return out
 

@@ -72,7 +72,12 @@ mst_status fail(mst_status s, const char* fmt, ...) {
     } while (0)
 
 // device-counter slots
-enum { C_ERR = 0, C_OUT = 1, C_NNEXT = 2, C_TILE = 3, C_ANEXT = 5 };  // C_TILE: 2 slots
+enum { C_ERR = 0, C_OUT = 1, C_NNEXT = 2, C_TILE = 3, C_AREC = 8 };  // C_TILE: 2 slots
+// C_AREC: per shard j and round r, the alive arcs entering round r (written by round r-1's
+// filter on the device; read back by the host together with n_{r+1} after the hook)
+constexpr int AREC_STRIDE = MST_MAX_ROUNDS + 1;
+inline int arec(int j, int r) { return C_AREC + j * AREC_STRIDE + r; }
+constexpr int DCNT_WORDS = C_AREC + 64 * AREC_STRIDE;
 
 struct Shard {
     u64 lo, hi;  // arc range [lo, hi) in arcs_0 and in the ping-pong buffers
@@ -249,14 +254,14 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     u32* cursor;
     CKS(galloc(g, &deg, n));
     CKS(galloc(g, &cursor, n));
-    CKS(galloc(g, &g->dcnt, 8 + 64));
+    CKS(galloc(g, &g->dcnt, DCNT_WORDS));
     CKS(galloc(g, &g->acc, 4));
     const u64 nslots = status_slots_needed(n, 2 * m, g->nwords);
     CKS(galloc(g, &g->status, nslots));
     CK(cudaMemsetAsync(g->status, 0, nslots * sizeof(u64), g->cst));
     CK(cudaMemsetAsync(deg, 0, std::max<u64>(n, 1) * sizeof(u32), g->cst));
-    CK(cudaMemsetAsync(g->dcnt, 0, 72 * sizeof(u32), g->cst));
-    CK(cudaMallocHost(&g->hcnt, 72 * sizeof(u32)));
+    CK(cudaMemsetAsync(g->dcnt, 0, DCNT_WORDS * sizeof(u32), g->cst));
+    CK(cudaMallocHost(&g->hcnt, DCNT_WORDS * sizeof(u32)));
     CK(cudaMallocHost(&g->hacc, 4 * sizeof(u64)));
 
     CK(launch_degree(g->cst, g->nsm, (u32)n, (u32)m, src, dst, g->eu, g->ev, deg, g->dcnt + C_ERR));
@@ -264,6 +269,17 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CK(cudaStreamSynchronize(g->cst));
     if (g->hcnt[0]) return fail(MST_EINVAL, "an endpoint is outside [0, n) (n = %lld)", (long long)n);
 
+    const char* ro = getenv("MST_REORDER");  // "0": keep the caller's vertex numbering
+    if (n > 0 && !(ro && ro[0] == '0')) {
+        // A0 locality layout: hub-first internal numbering (stable, by log2 degree)
+        u32 *degn, *newid, *counts;
+        CKS(galloc(g, &degn, n));
+        CKS(galloc(g, &newid, n));
+        CKS(galloc(g, &counts, reorder_scratch(n)));
+        CK(launch_reorder(g->cst, g->nsm, (u32)n, (u32)m, deg, degn, g->eu, g->ev, newid, counts,
+                          g->status, g->epoch++));
+        deg = degn;
+    }
     if (n > 0) {
         CK(launch_scan_rows(g->cst, (u32)n, deg, g->row, cursor, g->status, g->epoch++));
     } else {
@@ -397,7 +413,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         u64* tgt = g->sim ? g->shard_best + (u64)j * n : g->bestA;
         if (sh.A == 0) continue;
         Prof p(g, s, MST_K_MIN0, 0);
-        CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, g->dcnt + C_TILE, g->pass_seq++));
+        CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, (u32)n, g->dcnt + C_TILE,
+                       g->pass_seq++));
     }
     if (g->sim) {
         Prof p(g, s, MST_K_COMM, 0);
@@ -407,6 +424,11 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         CKN(ncclAllReduce(g->bestA, g->bestA, n, ncclUint64, ncclMin, g->comm, s));
     }
 
+    // round-0 arc counts (host-known) into the per-round record
+    for (int j = 0; j < G; ++j) g->hcnt[arec(j, 0)] = g->shards[j].A;
+    for (int j = 0; j < G; ++j)
+        CK(cudaMemcpyAsync(g->dcnt + arec(j, 0), g->hcnt + arec(j, 0), sizeof(u32),
+                           cudaMemcpyHostToDevice, s));
     MapChain chain;
     chain.len = 0;
     u64 moff = 0;
@@ -414,85 +436,84 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     u64* bcur = g->bestA;
     u64* bnxt = g->bestB;
     int r = 0, outb = 0;
-    bool first = true;
     bool dense = false;  // this round's alive arcs live in the min-matrix g->mat[mc]
     int mc = 0;
     g->st.dense_round = -1;
     while (true) {
         if (r >= MST_MAX_ROUNDS || chain.len >= MST_CHAIN_MAX)
             return fail(MST_EINTERNAL, "round limit exceeded (r = %d)", r);
-        u64 asum = 0;
-        for (auto& sh : g->shards) asum += sh.A;
-        g->st.n_r[r] = nr;
-        g->st.a_r[r] = dense ? (int64_t)dense_entries(nr) : (int64_t)asum;
         int* Mr = g->maps + moff;
         {
             Prof p(g, s, MST_K_HOOK, r);
             CK(launch_hook(s, nr, bcur, bnxt, g->eu, g->ev, chain, g->P, g->Mtmp, g->msf, g->acc,
                            g->status, g->epoch++, g->dcnt + C_NNEXT));
         }
+        // one host round trip per round: n_{r+1} (sizes round r's filter)
+        // and the arcs entering round r (written by round r-1's filter)
+        CK(cudaMemcpyAsync(g->hcnt + C_NNEXT, g->dcnt + C_NNEXT, sizeof(u32), cudaMemcpyDeviceToHost, s));
+        if (!dense)
+            for (int j = 0; j < G; ++j)
+                CK(cudaMemcpyAsync(g->hcnt + arec(j, r), g->dcnt + arec(j, r), sizeof(u32),
+                                   cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        const u32 nn = g->hcnt[C_NNEXT];
+        u64 asum = 0;
+        if (!dense)
+            for (int j = 0; j < G; ++j) {
+                g->shards[j].A = g->hcnt[arec(j, r)];
+                asum += g->shards[j].A;
+            }
+        g->st.n_r[r] = nr;
+        g->st.a_r[r] = dense ? (int64_t)dense_entries(nr) : (int64_t)asum;
+        if (nn <= 1) {  // <= 1 live component left: no inter-component edge remains
+            ++r;
+            break;
+        }
+        if (moff + nr + nn > 2 * n + 1) return fail(MST_EINTERNAL, "label-map storage overflow");
         {
             Prof p(g, s, MST_K_JUMP, r);
             CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, Mr));
         }
+        bool to_dense = false;
         if (dense) {
             // A9/NEXT-1 dense round: scan the matrix, collapse into the next (smaller) one
             Prof p(g, s, MST_K_DENSE, r);
-            CK(launch_dense_init(s, g->nsm, g->dcnt + C_NNEXT, g->mat[mc ^ 1]));
-            CK(launch_dense_round(s, g->nsm, nr, g->mat[mc], Mr, g->dcnt + C_NNEXT, g->mat[mc ^ 1],
-                                  bnxt));
+            CK(launch_dense_init(s, g->nsm, nn, g->mat[mc ^ 1]));
+            CK(launch_dense_round(s, g->nsm, nr, g->mat[mc], Mr, nn, g->mat[mc ^ 1], bnxt));
         } else {
-            if (g->mat[0]) CK(launch_dense_init(s, g->nsm, g->dcnt + C_NNEXT, g->mat[0]));
+            to_dense = g->mat[0] && nn <= (u32)DENSE_MAX;
+            if (to_dense) CK(launch_dense_init(s, g->nsm, nn, g->mat[0]));
             for (int j = 0; j < G; ++j) {
                 Shard& sh = g->shards[j];
                 u64* tgt = g->sim ? g->shard_best + (u64)j * n : bnxt;
-                if (sh.A == 0) {
-                    CK(cudaMemsetAsync(g->dcnt + C_ANEXT + j, 0, sizeof(u32), s));
-                    continue;
-                }
-                const uint4* in = (first ? g->arcs0 : g->abuf[outb ^ 1]) + sh.lo;
+                const uint4* in = (r == 0 ? g->arcs0 : g->abuf[outb ^ 1]) + sh.lo;
                 Prof p(g, s, MST_K_FILTER, r);
-                CK(launch_filter_min(s, g->nsm, sh.A, in, Mr, g->abuf[outb] + sh.lo, tgt,
-                                     g->dcnt + C_NNEXT, g->status, g->epoch++,
-                                     g->dcnt + C_ANEXT + j, g->dcnt + C_TILE, g->pass_seq++,
-                                     g->mat[0]));
+                CK(launch_filter_min(s, g->nsm, g->dcnt + arec(j, r), sh.A, in, Mr,
+                                     g->abuf[outb] + sh.lo, tgt, nn, g->status, g->epoch++,
+                                     g->dcnt + arec(j, r + 1), g->dcnt + C_TILE, g->pass_seq++,
+                                     to_dense ? g->mat[0] : nullptr));
             }
         }
-        CK(cudaMemcpyAsync(g->hcnt, g->dcnt, (C_ANEXT + G) * sizeof(u32), cudaMemcpyDeviceToHost, s));
-        CK(cudaStreamSynchronize(s));
-        const u32 nn = g->hcnt[C_NNEXT];
-        u64 anext = 0;
-        if (!dense) {
-            for (int j = 0; j < G; ++j) {
-                g->shards[j].A = g->hcnt[C_ANEXT + j];
-                anext += g->shards[j].A;
-            }
-        }
-        const bool was_dense = dense;
         chain.m[chain.len++] = Mr;
         moff += nr;
         ++r;
-        first = false;
         outb ^= 1;
-        if (nn <= 1) break;  // <= 1 live component: no inter-component edge is left
-        if (!dense && g->mat[0] && nn <= (u32)DENSE_MAX) {
-            dense = true;  // the filter just wrote the min-matrix g->mat[0]
+        if (g->sim && !dense) {
+            Prof p(g, s, MST_K_COMM, r);
+            CK(launch_combine_min(s, g->nsm, nn, G, g->shard_best, n, bnxt));
+        } else if (g->comm && !dense) {
+            Prof p(g, s, MST_K_COMM, r);
+            CKN(ncclAllReduce(bnxt, bnxt, nn, ncclUint64, ncclMin, g->comm, s));
+            if (to_dense)  // every rank needs the full matrix for the replicated dense rounds
+                CKN(ncclAllReduce(g->mat[0], g->mat[0], dense_entries(nn), ncclUint64, ncclMin,
+                                  g->comm, s));
+        }
+        if (to_dense) {
+            dense = true;
             mc = 0;
             g->st.dense_round = r;
         } else if (dense) {
             mc ^= 1;
-        }
-        if (!dense && !g->comm && anext == 0) break;
-        if (moff + nn > 2 * n + 1) return fail(MST_EINTERNAL, "label-map storage overflow");
-        if (g->sim && !was_dense) {
-            Prof p(g, s, MST_K_COMM, r);
-            CK(launch_combine_min(s, g->nsm, nn, G, g->shard_best, n, bnxt));
-        } else if (g->comm && !was_dense) {
-            Prof p(g, s, MST_K_COMM, r);
-            CKN(ncclAllReduce(bnxt, bnxt, nn, ncclUint64, ncclMin, g->comm, s));
-            if (dense)  // first dense round: every rank needs the full matrix
-                CKN(ncclAllReduce(g->mat[mc], g->mat[mc], dense_entries(nn), ncclUint64, ncclMin,
-                                  g->comm, s));
         }
         std::swap(bcur, bnxt);
         nr = nn;
@@ -686,7 +707,6 @@ mst_status mst_debug_filter_pass(mst_graph* g, mst_stream_t stream, int map_kind
         const u64 n = g->n;
         u32 ncomp = 0;
         CK(launch_debug_map(s, (u32)n, map_kind, (u32)group, g->maps, &ncomp));
-        CK(cudaMemcpyAsync(g->dcnt + C_NNEXT, &ncomp, sizeof(u32), cudaMemcpyHostToDevice, s));
         const Shard& sh = g->shards[0];
         const u32 A = (u32)(sh.hi - sh.lo);
         cudaEvent_t e0, e1;
@@ -695,9 +715,9 @@ mst_status mst_debug_filter_pass(mst_graph* g, mst_stream_t stream, int map_kind
         for (int it = -1; it < iters; ++it) {
             if (it == 0) CK(cudaEventRecord(e0, s));
             CK(cudaMemsetAsync(g->bestB, 0xff, n * sizeof(u64), s));
-            CK(launch_filter_min(s, g->nsm, A, g->arcs0 + sh.lo, g->maps, g->abuf[0] + sh.lo,
-                                 g->bestB, g->dcnt + C_NNEXT, g->status, g->epoch++,
-                                 g->dcnt + C_ANEXT, g->dcnt + C_TILE, g->pass_seq++, nullptr));
+            CK(launch_filter_min(s, g->nsm, nullptr, A, g->arcs0 + sh.lo, g->maps,
+                                 g->abuf[0] + sh.lo, g->bestB, ncomp, g->status, g->epoch++,
+                                 g->dcnt + arec(0, 1), g->dcnt + C_TILE, g->pass_seq++, nullptr));
         }
         CK(cudaEventRecord(e1, s));
         CK(cudaEventSynchronize(e1));
@@ -706,7 +726,7 @@ mst_status mst_debug_filter_pass(mst_graph* g, mst_stream_t stream, int map_kind
         cudaEventDestroy(e0);
         cudaEventDestroy(e1);
         u32 surv = 0;
-        CK(cudaMemcpy(&surv, g->dcnt + C_ANEXT, sizeof(u32), cudaMemcpyDeviceToHost));
+        CK(cudaMemcpy(&surv, g->dcnt + arec(0, 1), sizeof(u32), cudaMemcpyDeviceToHost));
         *out_ms = ms / iters;
         if (out_survivors) *out_survivors = surv;
         return MST_OK;
