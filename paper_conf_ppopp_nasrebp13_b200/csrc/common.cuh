@@ -151,6 +151,21 @@ __device__ __forceinline__ void run_min(u32 s, u32 hi, u32 lo, bool valid, u32 l
     ml = __reduce_min_sync(mask, v2);
 }
 
+// Warp-level duplicate collapse before an L2 min: lanes holding the same `cell` are grouped
+// with match.any, their keys are min-reduced through a per-warp shared scratch (32 x u64),
+// and only each group's leader issues the RED. Turns W identical-cell REDs into one.
+__device__ __forceinline__ void warp_dedup_red_min(u64* __restrict__ gbase, u32 cell, u64 key,
+                                                   bool active, u64* wslot, u32 lane) {
+    const u32 peers = __match_any_sync(FULL, active ? cell : 0xffffffffu);
+    const u32 leader = __ffs(peers) - 1;
+    if (lane == leader) wslot[lane] = KEY_INF;
+    __syncwarp();
+    if (active) red_min_shared(wslot + leader, key);
+    __syncwarp();
+    if (active && lane == leader) red_min_global(gbase + cell, wslot[lane]);
+    __syncwarp();
+}
+
 // tails of contiguous runs given their heads: lane l is a tail iff l == 31 or l+1 is a head
 __device__ __forceinline__ u32 run_tails(u32 heads) { return (heads >> 1) | 0x80000000u; }
 
