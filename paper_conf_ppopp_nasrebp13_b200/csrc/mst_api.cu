@@ -472,7 +472,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         if (moff + nr + nn > 2 * n + 1) return fail(MST_EINTERNAL, "label-map storage overflow");
         {
             Prof p(g, s, MST_K_JUMP, r);
-            CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, Mr));
+            CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, Mr, nn, bnxt));
         }
         bool to_dense = false;
         if (dense) {
