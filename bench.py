@@ -168,11 +168,9 @@ def run_gpu(args):
     ddst = torch.from_numpy(g.dst).cuda()
     dw = torch.from_numpy(g.w.view(np.int32)).cuda()
     if world > 1:
-        uid = torch.zeros(128, dtype=torch.uint8, device="cuda")
-        if rank == 0:
-            uid.copy_(torch.frombuffer(bytearray(mstb.mst_get_unique_id()), dtype=torch.uint8))
-        dist.broadcast(uid, 0)
-        h = mstb.MSTGraph(n, dsrc, ddst, dw, dist=(bytes(uid.cpu().numpy()), rank, world))
+        from paper_conf_ppopp_nasrebp13_b200 import dist as mdist
+        uid = mdist.share_unique_id(mstb.mst_get_unique_id)
+        h = mstb.MSTGraph(n, dsrc, ddst, dw, dist=(uid, rank, world))
     else:
         h = mstb.MSTGraph(n, dsrc, ddst, dw)
     del dsrc, ddst, dw
@@ -220,9 +218,8 @@ def run_gpu(args):
     clk = clocks.stop()
     total_ms = float(np.sum(step_ms))
     if world > 1:
-        t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms = float(t.item())
+        from paper_conf_ppopp_nasrebp13_b200 import dist as mdist
+        total_ms = mdist.max_over_ranks(total_ms)
     ids_np = ids.cpu().numpy()
     st = h.stats()
     peak, peak_src = measured_peaks()

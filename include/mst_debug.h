@@ -20,6 +20,16 @@ extern "C" {
 #endif
 mst_status mst_debug_filter_pass(mst_graph* g, mst_stream_t stream, int map_kind, int64_t group,
                                  int iters, double* out_ms, int64_t* out_survivors);
+
+/* mst_shard_ranges: the multi-GPU edge partition of mst_create_dist / mst_create_sim
+ * (SURVEY.md §8(e)), pure host code (no device needed):
+ *   row_offsets : HOST pointer, uint32[n+1], a CSR row-offset array (row[n] = arcs)
+ *   nranks      : 1..64 shards
+ *   lo, hi      : HOST int64[nranks]; shard j owns the arc window [lo[j], hi[j]), i.e. the
+ *                 sources [v_j, v_{j+1}) with v_j the first vertex whose offset reaches
+ *                 j * arcs / nranks. Windows are contiguous, disjoint and cover [0, arcs). */
+mst_status mst_shard_ranges(const uint32_t* row_offsets, int64_t n, int nranks, int64_t* lo,
+                            int64_t* hi);
 #ifdef __cplusplus
 }
 #endif

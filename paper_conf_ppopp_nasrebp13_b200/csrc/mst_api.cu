@@ -213,8 +213,25 @@ mst_status check_args(int64_t n, int64_t m, const void* src, const void* dst, co
     return MST_OK;
 }
 
-// Arc-balanced source ranges: shard g owns sources [v_g, v_{g+1}) with v_g the first vertex
-// whose row offset reaches g * A0 / G (computed from the CSR row offsets).
+// Arc-balanced source ranges: shard j owns the sources [v_j, v_{j+1}),
+// v_j = the first vertex whose CSR row offset reaches j * A0 / G; returns the arc windows
+// [row[v_j], row[v_{j+1}]). Pure host code (exported for tests as mst_shard_ranges).
+void compute_shard_ranges(const u32* row, u64 n, int G, u64* lo, u64* hi) {
+    const u64 A0 = row[n];
+    std::vector<u64> vb(G + 1);
+    vb[0] = 0;
+    vb[G] = n;
+    for (int j = 1; j < G; ++j) {
+        const u64 target = A0 * (u64)j / (u64)G;
+        vb[j] = (u64)(std::lower_bound(row, row + n + 1, (u32)target) - row);
+        vb[j] = std::min<u64>(std::max(vb[j], vb[j - 1]), n);
+    }
+    for (int j = 0; j < G; ++j) {
+        lo[j] = row[vb[j]];
+        hi[j] = row[vb[j + 1]];
+    }
+}
+
 mst_status shard_ranges(mst_graph* g, int G, std::vector<u64>& lo, std::vector<u64>& hi) {
     lo.assign(G, 0);
     hi.assign(G, 0);
@@ -226,19 +243,7 @@ mst_status shard_ranges(mst_graph* g, int G, std::vector<u64>& lo, std::vector<u
     CK(cudaMemcpyAsync(row.data(), g->row, (g->n + 1) * sizeof(u32), cudaMemcpyDeviceToHost,
                        g->cst));
     CK(cudaStreamSynchronize(g->cst));
-    std::vector<u64> vb(G + 1);
-    vb[0] = 0;
-    vb[G] = g->n;
-    for (int j = 1; j < G; ++j) {
-        const u64 target = g->A0 * (u64)j / (u64)G;
-        vb[j] = (u64)(std::lower_bound(row.begin(), row.end(), (u32)target) - row.begin());
-        vb[j] = std::max(vb[j], vb[j - 1]);
-        vb[j] = std::min<u64>(vb[j], g->n);
-    }
-    for (int j = 0; j < G; ++j) {
-        lo[j] = row[vb[j]];
-        hi[j] = row[vb[j + 1]];
-    }
+    compute_shard_ranges(row.data(), g->n, G, lo.data(), hi.data());
     return MST_OK;
 }
 
@@ -729,6 +734,21 @@ mst_status mst_debug_filter_pass(mst_graph* g, mst_stream_t stream, int map_kind
         CK(cudaMemcpy(&surv, g->dcnt + arec(0, 1), sizeof(u32), cudaMemcpyDeviceToHost));
         *out_ms = ms / iters;
         if (out_survivors) *out_survivors = surv;
+        return MST_OK;
+    });
+}
+
+mst_status mst_shard_ranges(const uint32_t* row_offsets, int64_t n, int nranks, int64_t* lo,
+                            int64_t* hi) {
+    return guarded([&]() -> mst_status {
+        if (!row_offsets || !lo || !hi || n < 0 || nranks < 1 || nranks > 64)
+            return fail(MST_EINVAL, "bad argument");
+        std::vector<u64> l(nranks), h(nranks);
+        compute_shard_ranges(row_offsets, (u64)n, nranks, l.data(), h.data());
+        for (int j = 0; j < nranks; ++j) {
+            lo[j] = (int64_t)l[j];
+            hi[j] = (int64_t)h[j];
+        }
         return MST_OK;
     });
 }

@@ -22,7 +22,7 @@ K_INIT, K_MIN0, K_HOOK, K_JUMP, K_FILTER, K_OUTPUT, K_COMM, K_DENSE, K_COUNT = r
 KERNEL_NAMES = ["init", "min0", "hook", "jump", "filter", "output", "comm", "dense"]
 
 # every symbol include/mst.h declares
-DEBUG_EXPORTS = ["mst_debug_filter_pass"]  # include/mst_debug.h (test/bench only)
+DEBUG_EXPORTS = ["mst_debug_filter_pass", "mst_shard_ranges"]  # include/mst_debug.h
 EXPORTS = ["mst_create", "mst_create_host", "mst_run", "mst_run_host", "mst_solve_host",
            "mst_destroy", "mst_last_error", "mst_get_stats", "mst_set_profiling",
            "mst_get_unique_id", "mst_create_dist", "mst_create_sim", "mst_version"]
@@ -85,6 +85,8 @@ def load(build_if_missing: bool = True):
     L.mst_debug_filter_pass.argtypes = [p, p, i32, i64, i32, ctypes.POINTER(ctypes.c_double),
                                         ctypes.POINTER(ctypes.c_int64)]
     L.mst_debug_filter_pass.restype = ctypes.c_int
+    L.mst_shard_ranges.argtypes = [p, i64, i32, p, p]
+    L.mst_shard_ranges.restype = ctypes.c_int
     for name in EXPORTS:
         if name not in ("mst_destroy", "mst_last_error", "mst_version"):
             getattr(L, name).restype = ctypes.c_int
@@ -233,6 +235,16 @@ def mst_solve_host(n, src, dst, w, out=None):
                                  dst.ctypes.data or None, w.ctypes.data or None,
                                  out.ctypes.data, ctypes.byref(cnt), ctypes.byref(tot)))
     return out[: cnt.value], int(cnt.value), int(tot.value)
+
+
+def mst_shard_ranges(row_offsets, nranks):
+    """The edge partition used by mst_create_dist (host only): arc windows (lo, hi) per rank."""
+    row = np.ascontiguousarray(row_offsets, np.uint32)
+    lo = np.empty(nranks, np.int64)
+    hi = np.empty(nranks, np.int64)
+    _check(load().mst_shard_ranges(row.ctypes.data, row.shape[0] - 1, int(nranks),
+                                   lo.ctypes.data, hi.ctypes.data))
+    return lo, hi
 
 
 def minimum_spanning_forest(n, src, dst, w, stream=None):
