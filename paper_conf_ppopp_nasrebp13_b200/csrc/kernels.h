@@ -25,6 +25,8 @@ cudaError_t launch_scan_rows(cudaStream_t st, u32 n, const u32* deg, u32* row, u
 cudaError_t launch_reorder(cudaStream_t st, int nsm, u32 n, u32 m, const u32* deg, u32* degn,
                            u32* eu, u32* ev, u32* newid, u32* counts, u64* status, u32 epoch);
 u64 reorder_scratch(u64 n);
+cudaError_t launch_owner_degree(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
+                                u32* odeg);
 cudaError_t launch_scatter(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
                            const unsigned* w, u32* cursor, uint4* arcs);
 cudaError_t launch_min0(cudaStream_t st, int nsm, u64 A, const uint4* arcs, u64* best, u32 nb,
@@ -33,7 +35,7 @@ cudaError_t launch_hook(cudaStream_t st, u32 nr, const u64* best, u64* best_next
                         const u32* ev, const MapChain& chain, u32* P, int* Mtmp, u32* msf,
                         u64* acc, u64* status, u32 epoch, u32* n_next);
 cudaError_t launch_jump(cudaStream_t st, int nsm, u32 nr, u32* P, const int* Mtmp, int* Mr,
-                        u32 nn, u64* best_next);
+                        const u32* nn, u64* best_next);
 cudaError_t launch_filter_min(cudaStream_t st, int nsm, const u32* a_in, u64 a_max,
                               const uint4* in, const int* M, uint4* out, u64* best, u32 nb,
                               u64* status, u32 epoch, u32* a_next, u32* tile_ctrs, u32 seq,

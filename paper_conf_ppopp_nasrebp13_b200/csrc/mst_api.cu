@@ -285,6 +285,13 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
                           g->status, g->epoch++));
         deg = degn;
     }
+    // owner degrees (each non-loop edge once, owned by its lower internal endpoint)
+    CK(cudaMemsetAsync(cursor, 0, std::max<u64>(n, 1) * sizeof(u32), g->cst));
+    CK(launch_owner_degree(g->cst, g->nsm, (u32)m, g->eu, g->ev, cursor));
+    deg = cursor;
+    u32* odeg_scan_out;
+    CKS(galloc(g, &odeg_scan_out, n));
+    cursor = odeg_scan_out;
     if (n > 0) {
         CK(launch_scan_rows(g->cst, (u32)n, deg, g->row, cursor, g->status, g->epoch++));
     } else {
@@ -453,6 +460,11 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             CK(launch_hook(s, nr, bcur, bnxt, g->eu, g->ev, chain, g->P, g->Mtmp, g->msf, g->acc,
                            g->status, g->epoch++, g->dcnt + C_NNEXT));
         }
+        {   // the jump does not need the host: it reads n_{r+1} on the device and runs
+            // while the counts travel to the host
+            Prof p(g, s, MST_K_JUMP, r);
+            CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, Mr, g->dcnt + C_NNEXT, bnxt));
+        }
         // one host round trip per round: n_{r+1} (sizes round r's filter)
         // and the arcs entering round r (written by round r-1's filter)
         CK(cudaMemcpyAsync(g->hcnt + C_NNEXT, g->dcnt + C_NNEXT, sizeof(u32), cudaMemcpyDeviceToHost, s));
@@ -475,10 +487,6 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             break;
         }
         if (moff + nr + nn > 2 * n + 1) return fail(MST_EINTERNAL, "label-map storage overflow");
-        {
-            Prof p(g, s, MST_K_JUMP, r);
-            CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, Mr, nn, bnxt));
-        }
         bool to_dense = false;
         if (dense) {
             // A9/NEXT-1 dense round: scan the matrix, collapse into the next (smaller) one
