@@ -23,7 +23,8 @@ cudaError_t launch_degree(cudaStream_t st, int nsm, u32 n, u32 m, const int* src
 cudaError_t launch_scan_rows(cudaStream_t st, u32 n, const u32* deg, u32* row, u32* cursor,
                              u64* status, u32 epoch);
 cudaError_t launch_reorder(cudaStream_t st, int nsm, u32 n, u32 m, const u32* deg, u32* degn,
-                           u32* eu, u32* ev, u32* newid, u32* counts, u64* status, u32 epoch);
+                           u32* eu, u32* ev, u32* newid, u32* counts, u64* status, u32 epoch,
+                           u32* odeg);
 u64 reorder_scratch(u64 n);
 cudaError_t launch_owner_degree(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
                                 u32* odeg);

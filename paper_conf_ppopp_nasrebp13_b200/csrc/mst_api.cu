@@ -274,20 +274,21 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CK(cudaStreamSynchronize(g->cst));
     if (g->hcnt[0]) return fail(MST_EINVAL, "an endpoint is outside [0, n) (n = %lld)", (long long)n);
 
+    // owner degrees (each non-loop edge once, owned by its lower internal endpoint)
+    CK(cudaMemsetAsync(cursor, 0, std::max<u64>(n, 1) * sizeof(u32), g->cst));
     const char* ro = getenv("MST_REORDER");  // "0": keep the caller's vertex numbering
     if (n > 0 && !(ro && ro[0] == '0')) {
-        // A0 locality layout: hub-first internal numbering (stable, by log2 degree)
+        // A0 locality layout: hub-first internal numbering (stable, by log2 degree); the
+        // relabelling pass also counts owner degrees in the new numbering
         u32 *degn, *newid, *counts;
         CKS(galloc(g, &degn, n));
         CKS(galloc(g, &newid, n));
         CKS(galloc(g, &counts, reorder_scratch(n)));
         CK(launch_reorder(g->cst, g->nsm, (u32)n, (u32)m, deg, degn, g->eu, g->ev, newid, counts,
-                          g->status, g->epoch++));
-        deg = degn;
+                          g->status, g->epoch++, cursor));
+    } else {
+        CK(launch_owner_degree(g->cst, g->nsm, (u32)m, g->eu, g->ev, cursor));
     }
-    // owner degrees (each non-loop edge once, owned by its lower internal endpoint)
-    CK(cudaMemsetAsync(cursor, 0, std::max<u64>(n, 1) * sizeof(u32), g->cst));
-    CK(launch_owner_degree(g->cst, g->nsm, (u32)m, g->eu, g->ev, cursor));
     deg = cursor;
     u32* odeg_scan_out;
     CKS(galloc(g, &odeg_scan_out, n));
