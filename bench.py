@@ -174,6 +174,10 @@ def run_gpu(args):
     else:
         h = mstb.MSTGraph(n, dsrc, ddst, dw)
     del dsrc, ddst, dw
+    if args.mode == "sparse":
+        h.set_option(mstb.mst.MST_OPT_DENSE, 0)
+    elif args.mode == "keep":
+        h.set_option(mstb.mst.MST_OPT_KEEP_EDGES, 1)
     build_ms = h.stats()["build_ms"]
     out_ids = torch.empty(max(n - 1, 1), dtype=torch.int32, device="cuda")
     stream = torch.cuda.current_stream()
@@ -268,7 +272,8 @@ def run_gpu(args):
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": total_ms / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
-            "config": {"workload": g.name, "n": n, "m": m, "arcs0": st["arcs0"],
+            "config": {"workload": g.name, "n": n, "m": m, "edge_records0": st["arcs0"],
+                       "mode": args.mode,
                        "rounds": st["rounds"], "seed": args.seed,
                        "generator": "graphgen (SURVEY.md §8(d) recipe)",
                        "l2": "flushed between timed steps (256 MB write); arcs > L2",
@@ -276,7 +281,7 @@ def run_gpu(args):
                        "build_ms": build_ms, "gen_s": gen_s},
             "parity": parity,
             "num_edges": cnt, "total_weight": tot,
-            "roofline": {"bound": "hbm", "kernel": "k_filter_min (A8)",
+            "roofline": {"bound": "hbm", "kernel": "k_arc_pass<MODE_FILTER> (A8)",
                          "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak if achieved else None, "traffic": traffic,
                          "peak_source": peak_src,
@@ -341,6 +346,9 @@ def main():
                     choices=["grid64", "uniform", "road", "rmat22", "dense"])
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--mode", default="morph", choices=["morph", "sparse", "keep"],
+                    help="morph: delete+compact, dense min-matrix at <= 4096 components "
+                         "(default); sparse: never dense; keep: the paper's no-deletion scheme")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-oracle", action="store_true")
     ap.add_argument("--ref-budget-s", type=float, default=150.0)

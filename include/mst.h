@@ -142,6 +142,21 @@ mst_status mst_get_stats(const mst_graph* g, mst_stats* out);
 /* enable (1) / disable (0) per-launch CUDA-event timing for subsequent runs */
 mst_status mst_set_profiling(mst_graph* g, int enable);
 
+/* ------------------------------------------------------------------ run options
+ * Options change how later mst_run calls work, never what they return (the forest is the
+ * unique F*, reading R1). MST_EINVAL for an unknown option or value.
+ *   MST_OPT_DENSE (default 1): once a round has <= 4096 live components, keep the alive
+ *       edges as a min-matrix over component pairs (duplicate collapse, SURVEY.md §8(a) A9 /
+ *       §8(f) NEXT-1); 0 = every round stays on the compacted edge list.
+ *   MST_OPT_KEEP_EDGES (default 0): 1 = the paper's own scheme ("maintains
+ *       the original adjacency list for each node and performs edge traversals per node"):
+ *       no deletion/compaction; every round re-reads all original edge records and skips
+ *       same-component ones through the explicitly maintained vertex->component map
+ *       (row A7). Implies MST_OPT_DENSE = 0. Used as an ablation of what the
+ *       morph step (deletion) buys. */
+enum { MST_OPT_DENSE = 1, MST_OPT_KEEP_EDGES = 2 };
+mst_status mst_set_option(mst_graph* g, int option, int64_t value);
+
 /* ------------------------------------------------------------------ multi-GPU (§8(e))
  * One process per GPU (torchrun). Every rank passes the identical full input; rank g keeps
  * the arcs whose source lies in its vertex range (ranges chosen from the CSR row offsets so

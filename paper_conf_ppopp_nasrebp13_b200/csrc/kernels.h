@@ -45,6 +45,7 @@ cudaError_t launch_dense_init(cudaStream_t st, int nsm, u32 n, u64* mat);
 cudaError_t launch_dense_round(cudaStream_t st, int nsm, u32 n, const u64* mat, const int* M,
                                u32 n_next, u64* mat_next, u64* best_next);
 u64 dense_entries(u64 n);
+cudaError_t launch_label_update(cudaStream_t st, int nsm, u32 n, int* L, const int* Mr, bool first);
 cudaError_t launch_output(cudaStream_t st, u32 nwords, const u32* msf, int* out, u64* status,
                           u32 epoch, u32* out_count);
 cudaError_t launch_combine_min(cudaStream_t st, int nsm, u32 nr, int nshards, u64* shard_best,

@@ -120,6 +120,10 @@ struct mst_graph {
     int rank = 0, nranks = 1;
     ncclComm_t comm = nullptr;
 
+    bool opt_dense = true;   // MST_OPT_DENSE
+    bool opt_keep = false;   // MST_OPT_KEEP_EDGES (paper-faithful ablation)
+    int* L = nullptr;        // vertex -> component labels (keep-edges mode, row A7)
+
     bool prof = false;
     std::vector<ProfRec> recs;
     std::vector<cudaEvent_t> evpool;
@@ -325,8 +329,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CKS(galloc(g, &g->Mtmp, n));
     CKS(galloc(g, &g->maps, 2 * n + 1));  // sum_r n_r <= 2n: every live component merges
     CKS(galloc(g, &g->msf, g->nwords));
-    const char* dz = getenv("MST_DENSE");  // "0": keep every round sparse (tests, ablation)
-    if (n >= 2 && !(dz && dz[0] == '0')) {  // dense min-matrices (A9 / NEXT-1), <= 67 MB each
+    if (n >= 2) {  // dense min-matrices (A9 / NEXT-1), <= 67 MB each
         CKS(galloc(g, &g->mat[0], dense_entries(n)));
         CKS(galloc(g, &g->mat[1], dense_entries(n)));
     }
@@ -495,13 +498,25 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             CK(launch_dense_init(s, g->nsm, nn, g->mat[mc ^ 1]));
             CK(launch_dense_round(s, g->nsm, nr, g->mat[mc], Mr, nn, g->mat[mc ^ 1], bnxt));
         } else {
-            to_dense = g->mat[0] && nn <= (u32)DENSE_MAX;
+            to_dense = g->mat[0] && g->opt_dense && !g->opt_keep && nn <= (u32)DENSE_MAX;
             if (to_dense) CK(launch_dense_init(s, g->nsm, nn, g->mat[0]));
+            if (g->opt_keep) {  // A7: the vertex -> component map, explicitly
+                Prof p(g, s, MST_K_JUMP, r);
+                CK(launch_label_update(s, g->nsm, (u32)n, g->L, Mr, r == 0));
+            }
             for (int j = 0; j < G; ++j) {
                 Shard& sh = g->shards[j];
                 u64* tgt = g->sim ? g->shard_best + (u64)j * n : bnxt;
-                const uint4* in = (r == 0 ? g->arcs0 : g->abuf[outb ^ 1]) + sh.lo;
                 Prof p(g, s, MST_K_FILTER, r);
+                if (g->opt_keep) {
+                    // the paper's scheme: every original record, every round
+                    const u64 A0j = sh.hi - sh.lo;
+                    CK(launch_filter_min(s, g->nsm, nullptr, A0j, g->arcs0 + sh.lo, g->L, nullptr,
+                                         tgt, nn, g->status, g->epoch++, g->dcnt + arec(j, r + 1),
+                                         g->dcnt + C_TILE, g->pass_seq++, nullptr));
+                    continue;
+                }
+                const uint4* in = (r == 0 ? g->arcs0 : g->abuf[outb ^ 1]) + sh.lo;
                 CK(launch_filter_min(s, g->nsm, g->dcnt + arec(j, r), sh.A, in, Mr,
                                      g->abuf[outb] + sh.lo, tgt, nn, g->status, g->epoch++,
                                      g->dcnt + arec(j, r + 1), g->dcnt + C_TILE, g->pass_seq++,
@@ -703,6 +718,25 @@ mst_status mst_get_stats(const mst_graph* g, mst_stats* out) {
     if (!g || !out) return fail(MST_EINVAL, "null argument");
     *out = g->st;
     return MST_OK;
+}
+
+mst_status mst_set_option(mst_graph* g, int option, int64_t value) {
+    return guarded([&]() -> mst_status {
+        if (!g) return fail(MST_EINVAL, "handle is NULL");
+        if (value != 0 && value != 1) return fail(MST_EINVAL, "option value must be 0 or 1");
+        if (option == MST_OPT_DENSE) {
+            g->opt_dense = value != 0;
+        } else if (option == MST_OPT_KEEP_EDGES) {
+            if (value && !g->L && g->n > 0) {
+                CKS(galloc(g, &g->L, g->n));
+                CK(cudaStreamSynchronize(g->cst));
+            }
+            g->opt_keep = value != 0;
+        } else {
+            return fail(MST_EINVAL, "unknown option %d", option);
+        }
+        return MST_OK;
+    });
 }
 
 mst_status mst_set_profiling(mst_graph* g, int enable) {

@@ -25,7 +25,9 @@ KERNEL_NAMES = ["init", "min0", "hook", "jump", "filter", "output", "comm", "den
 DEBUG_EXPORTS = ["mst_debug_filter_pass", "mst_shard_ranges"]  # include/mst_debug.h
 EXPORTS = ["mst_create", "mst_create_host", "mst_run", "mst_run_host", "mst_solve_host",
            "mst_destroy", "mst_last_error", "mst_get_stats", "mst_set_profiling",
-           "mst_get_unique_id", "mst_create_dist", "mst_create_sim", "mst_version"]
+           "mst_get_unique_id", "mst_create_dist", "mst_create_sim", "mst_version",
+           "mst_set_option"]
+MST_OPT_DENSE, MST_OPT_KEEP_EDGES = 1, 2
 
 
 class mst_stats(ctypes.Structure):
@@ -80,6 +82,7 @@ def load(build_if_missing: bool = True):
     L.mst_last_error.restype = ctypes.c_char_p
     L.mst_get_stats.argtypes = [p, ctypes.POINTER(mst_stats)]
     L.mst_set_profiling.argtypes = [p, i32]
+    L.mst_set_option.argtypes = [p, i32, i64]
     L.mst_get_unique_id.argtypes = [p]
     L.mst_version.restype = ctypes.c_char_p
     L.mst_debug_filter_pass.argtypes = [p, p, i32, i64, i32, ctypes.POINTER(ctypes.c_double),
@@ -176,6 +179,10 @@ class MSTGraph:
         _check(load().mst_run_host(self._h, _stream_ptr(stream), out.ctypes.data,
                                    ctypes.byref(cnt), ctypes.byref(tot)))
         return out[: cnt.value], int(cnt.value), int(tot.value)
+
+    def set_option(self, option: int, value: int):
+        """mst_set_option: MST_OPT_DENSE / MST_OPT_KEEP_EDGES (include/mst.h)."""
+        _check(load().mst_set_option(self._h, int(option), int(value)))
 
     def set_profiling(self, on: bool):
         _check(load().mst_set_profiling(self._h, 1 if on else 0))

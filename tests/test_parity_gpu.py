@@ -28,11 +28,13 @@ def dev(a, dt=torch.int32):
     return torch.from_numpy(a.astype(np.int32, copy=False)).to("cuda")
 
 
-def gpu_msf(lib, n, src, dst, w, nshards=1, runs=1):
+def gpu_msf(lib, n, src, dst, w, nshards=1, runs=1, options=()):
     src = np.asarray(src, np.int32)
     dst = np.asarray(dst, np.int32)
     w = np.asarray(w, np.uint64).astype(np.uint32)
     with lib.MSTGraph(n, dev(src), dev(dst), dev(w), nshards=nshards) as g:
+        for opt, val in options:
+            g.set_option(opt, val)
         outs = []
         for _ in range(runs):
             ids, cnt, tot = g.run()
@@ -43,8 +45,8 @@ def gpu_msf(lib, n, src, dst, w, nshards=1, runs=1):
     return outs[0][0], outs[0][1], outs[0][2], st
 
 
-def assert_parity(lib, oracle_mod, n, src, dst, w, nshards=1, runs=1):
-    ids, cnt, tot, st = gpu_msf(lib, n, src, dst, w, nshards, runs)
+def assert_parity(lib, oracle_mod, n, src, dst, w, nshards=1, runs=1, options=()):
+    ids, cnt, tot, st = gpu_msf(lib, n, src, dst, w, nshards, runs, options)
     o_ids, o_tot = oracle_mod.kruskal(n, src, dst, w)
     assert cnt == len(o_ids), (cnt, len(o_ids))
     assert tot == o_tot, (tot, o_tot)
@@ -206,12 +208,35 @@ def test_full_size_configs(lib, oracle_mod, gg, k):
 
 # ------------------------------------------------------------------ sparse-only rounds
 @pytest.mark.parametrize("k,sd", [(1, 0), (2, 6), (4, 8), (5, 6)])
-def test_sparse_only_rounds(lib, oracle_mod, gg, k, sd, monkeypatch):
-    """MST_DENSE=0 keeps every round on the compaction path (no dense min-matrix)."""
-    monkeypatch.setenv("MST_DENSE", "0")
+def test_sparse_only_rounds(lib, oracle_mod, gg, k, sd):
+    """MST_OPT_DENSE = 0 keeps every round on the compaction path (no dense min-matrix)."""
     g = gg.config(k, s=2, scale_down=sd)
-    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w)
+    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w,
+                       options=[(lib.mst.MST_OPT_DENSE, 0)], runs=2)
     assert st["dense_round"] == -1
+
+
+@pytest.mark.parametrize("k,sd", [(1, 0), (2, 6), (3, 8), (4, 8), (5, 6)])
+def test_keep_edges_paper_scheme(lib, oracle_mod, gg, k, sd):
+    """MST_OPT_KEEP_EDGES = 1: no deletion, original records re-read every round."""
+    g = gg.config(k, s=4, scale_down=sd)
+    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w,
+                       options=[(lib.mst.MST_OPT_KEEP_EDGES, 1)], runs=2)
+    assert st["dense_round"] == -1
+    assert all(a == st["arcs0"] for a in st["a_r"])  # nothing is ever deleted
+
+
+def test_options_switch_on_one_handle(lib, oracle_mod, gg):
+    g = gg.config(4, s=5, scale_down=8)
+    o_ids, o_tot = oracle_mod.kruskal(g.n, g.src, g.dst, g.w)
+    with lib.MSTGraph(g.n, dev(g.src), dev(g.dst), dev(g.w)) as h:
+        for opts in ([], [(2, 1)], [(2, 0), (1, 0)], [(1, 1)]):
+            for o, v in opts:
+                h.set_option(o, v)
+            ids, cnt, tot = h.run()
+            assert np.array_equal(ids.cpu().numpy(), o_ids) and tot == o_tot
+        with pytest.raises(lib.MSTError):
+            h.set_option(99, 1)
 
 
 @pytest.mark.parametrize("k,sd", [(1, 0), (4, 6), (5, 6)])

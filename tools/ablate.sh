@@ -1,7 +1,7 @@
 # usage: ENVS="A=1 B=2;C=3" bash tools/ablate.sh   (each ;-separated group is one run)
 IFS=';' read -ra GROUPS_ <<< "${ENVS:-X=0}"
 for grp in "${GROUPS_[@]}"; do
-  env $grp timeout 300 python bench.py --steps ${STEPS:-5} --warmup 3 --e2e-steps 0 --no-oracle --workload ${WL:-rmat22} > /tmp/ab.json 2> /tmp/ab.err
+  env $grp timeout 300 python bench.py --steps ${STEPS:-5} --warmup 3 --e2e-steps 0 --no-oracle --workload ${WL:-rmat22} --mode ${MODE:-morph} > /tmp/ab.json 2> /tmp/ab.err
   python -c "
 import json,sys
 try:
