@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 
 #define MST_CHAIN_MAX 64
+#define ACC_SLOTS 64  // forest weight/size accumulators: 64 (sum, count) pairs summed on the host
 #define DENSE_MAX 4096  // components: the dense min-matrix then holds <= 8.4 M entries (67 MB)
 
 namespace mstk {
@@ -29,11 +30,11 @@ u64 reorder_scratch(u64 n);
 cudaError_t launch_owner_degree(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
                                 u32* odeg);
 cudaError_t launch_scatter(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
-                           const unsigned* w, u32* cursor, uint4* arcs);
+                           const unsigned* w, u32* cursor, uint4* arcs, uint2* euv);
 cudaError_t launch_min0(cudaStream_t st, int nsm, u64 A, const uint4* arcs, u64* best, u32 nb,
                         u32* tile_ctrs, u32 seq);
-cudaError_t launch_hook(cudaStream_t st, u32 nr, const u64* best, u64* best_next, const u32* eu,
-                        const u32* ev, const MapChain& chain, u32* P, int* Mtmp, u32* msf,
+cudaError_t launch_hook(cudaStream_t st, u32 nr, const u64* best, u64* best_next, u64* hmap, u32 tag,
+                        const uint2* euv, const MapChain& chain, u32* P, int* Mtmp, u32* msf,
                         u64* acc, u64* status, u32 epoch, u32* n_next);
 cudaError_t launch_jump(cudaStream_t st, int nsm, u32 nr, u32* P, const int* Mtmp, int* Mr,
                         const u32* nn, u64* best_next);

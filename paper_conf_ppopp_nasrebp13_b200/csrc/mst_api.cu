@@ -99,6 +99,7 @@ struct mst_graph {
     std::vector<void*> allocs;
 
     u32 *eu = nullptr, *ev = nullptr, *row = nullptr;
+    uint2* euv = nullptr;  // {eu, ev} interleaved: the hook's partner lookup
     uint4* arcs0 = nullptr;                 // A_0 arcs {s, d, eid, w}, grouped by source
     uint4* abuf[2] = {nullptr, nullptr};    // ping-pong alive arcs of rounds >= 1
     u64 *bestA = nullptr, *bestB = nullptr, *shard_best = nullptr;
@@ -112,6 +113,9 @@ struct mst_graph {
     u32* dcnt = nullptr;
     u64* acc = nullptr;
     u32* hcnt = nullptr;  // pinned
+    volatile u64* hmap = nullptr;  // pinned + mapped: tagged n_{r+1} written by the hook
+    u64* dmap = nullptr;           // its device alias
+    u32 run_seq = 0;
     u64* hacc = nullptr;  // pinned
     int* out_tmp = nullptr;  // for mst_run_host
 
@@ -171,6 +175,7 @@ void release(mst_graph* g) {
     }
     if (g->hcnt) cudaFreeHost(g->hcnt);
     if (g->hacc) cudaFreeHost(g->hacc);
+    if (g->hmap) cudaFreeHost((void*)g->hmap);
     for (auto e : g->evpool) cudaEventDestroy(e);
     if (g->cst) cudaStreamDestroy(g->cst);
     delete g;
@@ -264,14 +269,21 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CKS(galloc(g, &deg, n));
     CKS(galloc(g, &cursor, n));
     CKS(galloc(g, &g->dcnt, DCNT_WORDS));
-    CKS(galloc(g, &g->acc, 4));
+    CKS(galloc(g, &g->acc, 2 * ACC_SLOTS));
     const u64 nslots = status_slots_needed(n, 2 * m, g->nwords);
     CKS(galloc(g, &g->status, nslots));
     CK(cudaMemsetAsync(g->status, 0, nslots * sizeof(u64), g->cst));
     CK(cudaMemsetAsync(deg, 0, std::max<u64>(n, 1) * sizeof(u32), g->cst));
     CK(cudaMemsetAsync(g->dcnt, 0, DCNT_WORDS * sizeof(u32), g->cst));
     CK(cudaMallocHost(&g->hcnt, DCNT_WORDS * sizeof(u32)));
-    CK(cudaMallocHost(&g->hacc, 4 * sizeof(u64)));
+    CK(cudaMallocHost(&g->hacc, 2 * ACC_SLOTS * sizeof(u64)));
+    {
+        void* hm = nullptr;
+        CK(cudaHostAlloc(&hm, (MST_MAX_ROUNDS + 1) * sizeof(u64), cudaHostAllocMapped));
+        memset(hm, 0, (MST_MAX_ROUNDS + 1) * sizeof(u64));
+        g->hmap = (volatile u64*)hm;
+        CK(cudaHostGetDevicePointer((void**)&g->dmap, hm, 0));
+    }
 
     CK(launch_degree(g->cst, g->nsm, (u32)n, (u32)m, src, dst, g->eu, g->ev, deg, g->dcnt + C_ERR));
     CK(cudaMemcpyAsync(g->hcnt, g->dcnt, sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
@@ -307,7 +319,8 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CK(cudaStreamSynchronize(g->cst));
     g->A0 = A0;
     CKS(galloc(g, &g->arcs0, A0));
-    CK(launch_scatter(g->cst, g->nsm, (u32)m, g->eu, g->ev, w, cursor, g->arcs0));
+    CKS(galloc(g, &g->euv, m));
+    CK(launch_scatter(g->cst, g->nsm, (u32)m, g->eu, g->ev, w, cursor, g->arcs0, g->euv));
 
     // shards: simulation = all G ranges locally; distributed = this rank's range only
     const int G = nshards_sim > 1 ? nshards_sim : nranks;
@@ -391,6 +404,34 @@ mst_status create_common(int64_t n, int64_t m, const int32_t* src, const int32_t
 }
 
 // --------------------------------------------------------------------------- run
+// Spin on the tagged word the hook writes to mapped host memory (no memcpy, no stream sync);
+// a failing kernel never writes it, so the stream is queried now and then for errors.
+mst_status wait_round(mst_graph* g, cudaStream_t s, int r, u32 tag, u32* nn) {
+    const auto t0 = std::chrono::steady_clock::now();
+    for (u64 spin = 0;; ++spin) {
+        const u64 v = g->hmap[r];
+        if ((u32)(v >> 32) == tag) {
+            *nn = (u32)v;
+            return MST_OK;
+        }
+        if ((spin & 1023) == 1023) {
+            const cudaError_t e = cudaStreamQuery(s);
+            if (e != cudaSuccess && e != cudaErrorNotReady)
+                return fail(MST_ECUDA, "round %d: %s", r, cudaGetErrorString(e));
+            if (e == cudaSuccess) {  // stream drained: the word must be visible now
+                const u64 w = g->hmap[r];
+                if ((u32)(w >> 32) == tag) {
+                    *nn = (u32)w;
+                    return MST_OK;
+                }
+                return fail(MST_EINTERNAL, "round %d: size word not written", r);
+            }
+            if (std::chrono::steady_clock::now() - t0 > std::chrono::seconds(120))
+                return fail(MST_EINTERNAL, "round %d: timed out waiting for the hook", r);
+        }
+    }
+}
+
 mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out_num,
                     uint64_t* out_total) {
     const u64 n = g->n;
@@ -419,7 +460,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         Prof p(g, s, MST_K_INIT, 0);
         CK(cudaMemsetAsync(g->bestA, 0xff, n * sizeof(u64), s));
         CK(cudaMemsetAsync(g->msf, 0, std::max<u64>(g->nwords, 1) * sizeof(u32), s));
-        CK(cudaMemsetAsync(g->acc, 0, 4 * sizeof(u64), s));
+        CK(cudaMemsetAsync(g->acc, 0, 2 * ACC_SLOTS * sizeof(u64), s));
         if (g->sim) CK(cudaMemsetAsync(g->shard_best, 0xff, n * G * sizeof(u64), s));
     }
     // ---- A2 round-0 minimum (+ A3)
@@ -445,6 +486,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     for (int j = 0; j < G; ++j)
         CK(cudaMemcpyAsync(g->dcnt + arec(j, 0), g->hcnt + arec(j, 0), sizeof(u32),
                            cudaMemcpyHostToDevice, s));
+    const u32 tag_base = ((++g->run_seq) & 0xffffffu) << 8;  // run-unique tags for hmap
     MapChain chain;
     chain.len = 0;
     u64 moff = 0;
@@ -461,7 +503,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         int* Mr = g->maps + moff;
         {
             Prof p(g, s, MST_K_HOOK, r);
-            CK(launch_hook(s, nr, bcur, bnxt, g->eu, g->ev, chain, g->P, g->Mtmp, g->msf, g->acc,
+            CK(launch_hook(s, nr, bcur, bnxt, g->dmap + r, tag_base | (u32)r, g->euv, chain, g->P, g->Mtmp, g->msf, g->acc,
                            g->status, g->epoch++, g->dcnt + C_NNEXT));
         }
         {   // the jump does not need the host: it reads n_{r+1} on the device and runs
@@ -469,23 +511,12 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             Prof p(g, s, MST_K_JUMP, r);
             CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, Mr, g->dcnt + C_NNEXT, bnxt));
         }
-        // one host round trip per round: n_{r+1} (sizes round r's filter)
-        // and the arcs entering round r (written by round r-1's filter)
-        CK(cudaMemcpyAsync(g->hcnt + C_NNEXT, g->dcnt + C_NNEXT, sizeof(u32), cudaMemcpyDeviceToHost, s));
-        if (!dense)
-            for (int j = 0; j < G; ++j)
-                CK(cudaMemcpyAsync(g->hcnt + arec(j, r), g->dcnt + arec(j, r), sizeof(u32),
-                                   cudaMemcpyDeviceToHost, s));
-        CK(cudaStreamSynchronize(s));
-        const u32 nn = g->hcnt[C_NNEXT];
-        u64 asum = 0;
-        if (!dense)
-            for (int j = 0; j < G; ++j) {
-                g->shards[j].A = g->hcnt[arec(j, r)];
-                asum += g->shards[j].A;
-            }
+        // one host round trip per round: n_{r+1} (sizes round r's filter),
+        // read zero-copy from the word the hook's last tile writes to mapped host memory
+        u32 nn;
+        CKS(wait_round(g, s, r, tag_base | (u32)r, &nn));
         g->st.n_r[r] = nr;
-        g->st.a_r[r] = dense ? (int64_t)dense_entries(nr) : (int64_t)asum;
+        g->st.a_r[r] = dense ? (int64_t)dense_entries(nr) : -1;  // sparse: filled at the end
         if (nn <= 1) {  // <= 1 live component left: no inter-component edge remains
             ++r;
             break;
@@ -548,6 +579,9 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         nr = nn;
     }
     g->st.rounds = r;
+    // per-round alive records (device-side counters, fetched once per run for the stats)
+    CK(cudaMemcpyAsync(g->hcnt + C_AREC, g->dcnt + C_AREC, (size_t)G * AREC_STRIDE * sizeof(u32),
+                       cudaMemcpyDeviceToHost, s));
     // ---- A11 output
     {
         Prof p(g, s, MST_K_OUTPUT, r);
@@ -559,8 +593,18 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         }
     }
     CK(cudaMemcpyAsync(g->hcnt, g->dcnt, 2 * sizeof(u32), cudaMemcpyDeviceToHost, s));
-    CK(cudaMemcpyAsync(g->hacc, g->acc, 2 * sizeof(u64), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(g->hacc, g->acc, 2 * ACC_SLOTS * sizeof(u64), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
+    for (int i = 1; i < ACC_SLOTS; ++i) {  // sum the spread accumulators
+        g->hacc[0] += g->hacc[2 * i];
+        g->hacc[1] += g->hacc[2 * i + 1];
+    }
+    for (int rr = 0; rr < r; ++rr) {
+        if (g->st.a_r[rr] >= 0) continue;
+        int64_t a = 0;
+        for (int j = 0; j < G; ++j) a += g->hcnt[arec(j, rr)];
+        g->st.a_r[rr] = a;
+    }
     if ((u64)g->hcnt[C_OUT] != g->hacc[1])
         return fail(MST_EINTERNAL, "forest size mismatch: %u ids vs %llu hooks", g->hcnt[C_OUT],
                     (unsigned long long)g->hacc[1]);
