@@ -102,6 +102,8 @@ __device__ __forceinline__ bool min_update(u64* p, u64 key) {
 __device__ __forceinline__ void red_min_global(u64* p, u64 key) {
     asm volatile("red.relaxed.gpu.global.min.u64 [%0], %1;" :: "l"(p), "l"(key) : "memory");
 }
+// (No native 64-bit shared min on sm_100a: this lowers to ATOMS.CAST.SPIN.64, measured faster
+// than an explicit read-then-CAS loop.)
 __device__ __forceinline__ void red_min_shared(u64* p, u64 key) {
     asm volatile("red.shared.min.u64 [%0], %1;" :: "r"((u32)__cvta_generic_to_shared(p)), "l"(key)
                  : "memory");
