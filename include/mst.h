@@ -65,8 +65,10 @@ typedef struct mst_graph mst_graph; /* opaque; owned by the library */
 mst_status mst_create(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                       const uint32_t* w, mst_graph** out);
 
-/* mst_create_host — as mst_create but src/dst/w are HOST pointers (pageable or pinned);
- * the library copies them to the device (input transferred to the GPU). */
+/* mst_create_host — as mst_create but src/dst/w are HOST pointers (pageable or pinned).
+ * Pinned (page-locked) arrays are read by the build kernels directly over PCIe (zero-copy,
+ * the transfer overlaps the validation and scatter passes); pageable arrays are first staged
+ * through a device copy (input transferred to the GPU). */
 mst_status mst_create_host(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                            const uint32_t* w, mst_graph** out);
 
@@ -92,7 +94,9 @@ mst_status mst_run_host(mst_graph* g, mst_stream_t stream, int32_t* out_edge_ids
 
 /* mst_solve_host — one end-to-end call from host arrays to host results:
  * mst_create_host + mst_run_host + mst_destroy. Device memory comes from a stream-ordered
- * pool that the library keeps between calls, so repeated solves do not pay cudaMalloc. */
+ * pool that the library keeps between calls, so repeated solves do not pay cudaMalloc. Being
+ * one-shot, it skips the build's hub-first relabelling pass (it costs more than one run
+ * saves); the result is identical. */
 mst_status mst_solve_host(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                           const uint32_t* w, int32_t* out_edge_ids_host,
                           int64_t* out_num_edges, uint64_t* out_total_weight);

@@ -257,7 +257,7 @@ mst_status shard_ranges(mst_graph* g, int G, std::vector<u64>& lo, std::vector<u
 }
 
 mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w, int nshards_sim,
-                 int rank, int nranks) {
+                 int rank, int nranks, bool reorder) {
     auto t0 = std::chrono::steady_clock::now();
     const u64 n = g->n, m = g->m;
     g->nwords = (m + 31) / 32;
@@ -293,7 +293,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     // owner degrees (each non-loop edge once, owned by its lower internal endpoint)
     CK(cudaMemsetAsync(cursor, 0, std::max<u64>(n, 1) * sizeof(u32), g->cst));
     const char* ro = getenv("MST_REORDER");  // "0": keep the caller's vertex numbering
-    if (n > 0 && !(ro && ro[0] == '0')) {
+    if (n > 0 && reorder && !(ro && ro[0] == '0')) {
         // A0 locality layout: hub-first internal numbering (stable, by log2 degree); the
         // relabelling pass also counts owner degrees in the new numbering
         u32 *degn, *newid, *counts;
@@ -362,7 +362,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
 
 mst_status create_common(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                          const uint32_t* w, int nshards_sim, const uint8_t* id, int rank,
-                         int nranks, mst_graph** out) {
+                         int nranks, mst_graph** out, bool reorder = true) {
     if (!out) return fail(MST_EINVAL, "out is NULL");
     *out = nullptr;
     CKS(check_args(n, m, src, dst, w));
@@ -385,7 +385,7 @@ mst_status create_common(int64_t n, int64_t m, const int32_t* src, const int32_t
         release(g);
         return fail(MST_ECUDA, "device setup: %s", cudaGetErrorString(e));
     }
-    mst_status s = build(g, src, dst, (const unsigned*)w, nshards_sim, rank, nranks);
+    mst_status s = build(g, src, dst, (const unsigned*)w, nshards_sim, rank, nranks, reorder);
     if (s == MST_OK && nranks > 1) {
         ncclUniqueId uid;
         memcpy(&uid, id, sizeof uid);
@@ -677,40 +677,64 @@ mst_status mst_create_dist(int64_t n, int64_t m, const int32_t* src, const int32
     });
 }
 
+// Host-array input. Pinned (page-locked) arrays are device-addressable under UVA: the build
+// kernels then read them straight over PCIe (zero-copy), so the transfer overlaps the
+// validation/degree and scatter passes instead of preceding them. Pageable arrays are staged
+// through a device copy first.
+static const void* device_alias(const void* p) {
+    cudaPointerAttributes a;
+    if (!p || cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        (void)cudaGetLastError();
+        return nullptr;
+    }
+    if (a.type == cudaMemoryTypeHost && a.devicePointer) return a.devicePointer;
+    if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) return p;
+    return nullptr;
+}
+
+static mst_status create_host_impl(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
+                                   const uint32_t* w, mst_graph** out, bool reorder) {
+    if (!out) return fail(MST_EINVAL, "out is NULL");
+    *out = nullptr;
+    CKS(check_args(n, m, src, dst, w));
+    int dev;
+    CK(cudaGetDevice(&dev));
+    CKS(configure_pool(dev));
+    if (m > 0) {
+        const void *as = device_alias(src), *ad = device_alias(dst), *aw = device_alias(w);
+        if (as && ad && aw)
+            return create_common(n, m, (const int32_t*)as, (const int32_t*)ad,
+                                 (const uint32_t*)aw, 1, nullptr, 0, 1, out, reorder);
+    }
+    cudaStream_t st;
+    CK(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+    void *ds = nullptr, *dd = nullptr, *dw = nullptr;
+    const size_t b = std::max<size_t>((size_t)m * 4, 16);
+    cudaError_t e = cudaMallocAsync(&ds, b, st);
+    if (e == cudaSuccess) e = cudaMallocAsync(&dd, b, st);
+    if (e == cudaSuccess) e = cudaMallocAsync(&dw, b, st);
+    if (e == cudaSuccess && m > 0) e = cudaMemcpyAsync(ds, src, (size_t)m * 4, cudaMemcpyHostToDevice, st);
+    if (e == cudaSuccess && m > 0) e = cudaMemcpyAsync(dd, dst, (size_t)m * 4, cudaMemcpyHostToDevice, st);
+    if (e == cudaSuccess && m > 0) e = cudaMemcpyAsync(dw, w, (size_t)m * 4, cudaMemcpyHostToDevice, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    mst_status s = MST_OK;
+    if (e != cudaSuccess)
+        s = fail(e == cudaErrorMemoryAllocation ? MST_ENOMEM : MST_ECUDA, "host->device input copy: %s",
+                 cudaGetErrorString(e));
+    else
+        s = create_common(n, m, (const int32_t*)ds, (const int32_t*)dd, (const uint32_t*)dw, 1,
+                          nullptr, 0, 1, out, reorder);
+    if (ds) cudaFreeAsync(ds, st);
+    if (dd) cudaFreeAsync(dd, st);
+    if (dw) cudaFreeAsync(dw, st);
+    cudaStreamSynchronize(st);
+    cudaStreamDestroy(st);
+    return s;
+}
+
 mst_status mst_create_host(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                            const uint32_t* w, mst_graph** out) {
-    return guarded([&]() -> mst_status {
-        if (!out) return fail(MST_EINVAL, "out is NULL");
-        *out = nullptr;
-        CKS(check_args(n, m, src, dst, w));
-        int dev;
-        CK(cudaGetDevice(&dev));
-        CKS(configure_pool(dev));
-        cudaStream_t st;
-        CK(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
-        void *ds = nullptr, *dd = nullptr, *dw = nullptr;
-        const size_t b = std::max<size_t>((size_t)m * 4, 16);
-        cudaError_t e = cudaMallocAsync(&ds, b, st);
-        if (e == cudaSuccess) e = cudaMallocAsync(&dd, b, st);
-        if (e == cudaSuccess) e = cudaMallocAsync(&dw, b, st);
-        if (e == cudaSuccess && m > 0) e = cudaMemcpyAsync(ds, src, (size_t)m * 4, cudaMemcpyHostToDevice, st);
-        if (e == cudaSuccess && m > 0) e = cudaMemcpyAsync(dd, dst, (size_t)m * 4, cudaMemcpyHostToDevice, st);
-        if (e == cudaSuccess && m > 0) e = cudaMemcpyAsync(dw, w, (size_t)m * 4, cudaMemcpyHostToDevice, st);
-        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-        mst_status s = MST_OK;
-        if (e != cudaSuccess)
-            s = fail(e == cudaErrorMemoryAllocation ? MST_ENOMEM : MST_ECUDA, "host->device input copy: %s",
-                     cudaGetErrorString(e));
-        else
-            s = create_common(n, m, (const int32_t*)ds, (const int32_t*)dd, (const uint32_t*)dw, 1,
-                              nullptr, 0, 1, out);
-        if (ds) cudaFreeAsync(ds, st);
-        if (dd) cudaFreeAsync(dd, st);
-        if (dw) cudaFreeAsync(dw, st);
-        cudaStreamSynchronize(st);
-        cudaStreamDestroy(st);
-        return s;
-    });
+    return guarded([&]() { return create_host_impl(n, m, src, dst, w, out, true); });
 }
 
 mst_status mst_run(mst_graph* g, mst_stream_t stream, int32_t* out_edge_ids,
@@ -747,7 +771,8 @@ mst_status mst_solve_host(int64_t n, int64_t m, const int32_t* src, const int32_
                           const uint32_t* w, int32_t* out_ids_host, int64_t* out_num_edges,
                           uint64_t* out_total_weight) {
     mst_graph* g = nullptr;
-    mst_status s = mst_create_host(n, m, src, dst, w, &g);
+    // one-shot: no hub-first relabelling (its build pass costs more than one run saves)
+    mst_status s = guarded([&]() { return create_host_impl(n, m, src, dst, w, &g, false); });
     if (s != MST_OK) return s;
     s = mst_run_host(g, g->cst, out_ids_host, out_num_edges, out_total_weight);
     std::string keep = g_err;

@@ -168,6 +168,14 @@ def test_host_paths(lib, oracle_mod, gg):
     with lib.MSTGraph(g.n, g.src, g.dst, g.w, host=True) as h:
         ids, cnt, tot = h.run_host()
         assert np.array_equal(ids, o_ids) and tot == o_tot
+    # pinned host arrays: the build reads them zero-copy over PCIe
+    pin = lambda a: torch.from_numpy(np.ascontiguousarray(a).view(np.int32)).pin_memory().numpy()  # noqa: E731
+    ps, pd, pw = pin(g.src), pin(g.dst), pin(g.w).view(np.uint32)
+    ids, cnt, tot = lib.mst_solve_host(g.n, ps, pd, pw)
+    assert np.array_equal(ids, o_ids) and tot == o_tot
+    with lib.MSTGraph(g.n, ps, pd, pw, host=True) as h:
+        ids, cnt, tot = h.run_host()
+        assert np.array_equal(ids, o_ids) and tot == o_tot
 
 
 def test_errors(lib):
