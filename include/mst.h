@@ -157,8 +157,11 @@ mst_status mst_set_profiling(mst_graph* g, int enable);
  *       no deletion/compaction; every round re-reads all original edge records and skips
  *       same-component ones through the explicitly maintained vertex->component map
  *       (row A7). Implies MST_OPT_DENSE = 0. Used as an ablation of what the
- *       morph step (deletion) buys. */
-enum { MST_OPT_DENSE = 1, MST_OPT_KEEP_EDGES = 2 };
+ *       morph step (deletion) buys.
+ *   MST_OPT_DEVICE_TAIL (default 1): once dense, run every remaining round inside one
+ *       cooperative kernel (no host round trip per round); 0 = one launch set per round.
+ */
+enum { MST_OPT_DENSE = 1, MST_OPT_KEEP_EDGES = 2, MST_OPT_DEVICE_TAIL = 3 };
 mst_status mst_set_option(mst_graph* g, int option, int64_t value);
 
 /* ------------------------------------------------------------------ multi-GPU (§8(e))

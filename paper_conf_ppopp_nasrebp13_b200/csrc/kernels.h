@@ -46,6 +46,9 @@ cudaError_t launch_dense_init(cudaStream_t st, int nsm, u32 n, u64* mat);
 cudaError_t launch_dense_round(cudaStream_t st, int nsm, u32 n, const u64* mat, const int* M,
                                u32 n_next, u64* mat_next, u64* best_next);
 u64 dense_entries(u64 n);
+cudaError_t launch_dense_tail(cudaStream_t st, int nsm, u32 n0, u64* best0, u64* best1,
+                              u64* mat0, u64* mat1, const uint2* euv, const MapChain& chain,
+                              u32* msf, u64* acc, u32* bar, u32* stats);
 cudaError_t launch_label_update(cudaStream_t st, int nsm, u32 n, int* L, const int* Mr, bool first);
 cudaError_t launch_output(cudaStream_t st, u32 nwords, const u32* msf, int* out, u64* status,
                           u32 epoch, u32* out_count);

@@ -77,7 +77,9 @@ enum { C_ERR = 0, C_OUT = 1, C_NNEXT = 2, C_TILE = 3, C_AREC = 8 };  // C_TILE: 
 // filter on the device; read back by the host together with n_{r+1} after the hook)
 constexpr int AREC_STRIDE = MST_MAX_ROUNDS + 1;
 inline int arec(int j, int r) { return C_AREC + j * AREC_STRIDE + r; }
-constexpr int DCNT_WORDS = C_AREC + 64 * AREC_STRIDE;
+constexpr int C_BAR = C_AREC + 64 * AREC_STRIDE;  // grid barrier {count, generation}
+constexpr int C_TAIL = C_BAR + 2;                   // device tail: rounds, n per round
+constexpr int DCNT_WORDS = C_TAIL + 1 + MST_MAX_ROUNDS;
 
 struct Shard {
     u64 lo, hi;  // arc range [lo, hi) in arcs_0 and in the ping-pong buffers
@@ -126,6 +128,7 @@ struct mst_graph {
 
     bool opt_dense = true;   // MST_OPT_DENSE
     bool opt_keep = false;   // MST_OPT_KEEP_EDGES (paper-faithful ablation)
+    bool opt_tail = true;    // MST_OPT_DEVICE_TAIL
     int* L = nullptr;        // vertex -> component labels (keep-edges mode, row A7)
 
     bool prof = false;
@@ -497,9 +500,18 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     bool dense = false;  // this round's alive arcs live in the min-matrix g->mat[mc]
     int mc = 0;
     g->st.dense_round = -1;
+    int tail_r0 = -1;  // first round run by the device-resident dense tail
     while (true) {
         if (r >= MST_MAX_ROUNDS || chain.len >= MST_CHAIN_MAX)
             return fail(MST_EINTERNAL, "round limit exceeded (r = %d)", r);
+        if (dense && g->opt_tail) {
+            // every remaining round in one cooperative launch (A4/A5/A6/A9 on the device)
+            Prof p(g, s, MST_K_DENSE, r);
+            CK(launch_dense_tail(s, g->nsm, nr, bcur, bnxt, g->mat[mc], g->mat[mc ^ 1], g->euv,
+                                 chain, g->msf, g->acc, g->dcnt + C_BAR, g->dcnt + C_TAIL));
+            tail_r0 = r;
+            break;
+        }
         int* Mr = g->maps + moff;
         {
             Prof p(g, s, MST_K_HOOK, r);
@@ -578,6 +590,9 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         std::swap(bcur, bnxt);
         nr = nn;
     }
+    if (tail_r0 >= 0)
+        CK(cudaMemcpyAsync(g->hcnt + C_TAIL, g->dcnt + C_TAIL, (1 + MST_MAX_ROUNDS) * sizeof(u32),
+                           cudaMemcpyDeviceToHost, s));
     g->st.rounds = r;
     // per-round alive records (device-side counters, fetched once per run for the stats)
     CK(cudaMemcpyAsync(g->hcnt + C_AREC, g->dcnt + C_AREC, (size_t)G * AREC_STRIDE * sizeof(u32),
@@ -598,6 +613,15 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     for (int i = 1; i < ACC_SLOTS; ++i) {  // sum the spread accumulators
         g->hacc[0] += g->hacc[2 * i];
         g->hacc[1] += g->hacc[2 * i + 1];
+    }
+    if (tail_r0 >= 0) {  // rounds run by the device tail
+        const u32 k = g->hcnt[C_TAIL];
+        for (u32 i = 0; i < k && tail_r0 + (int)i < MST_MAX_ROUNDS; ++i) {
+            g->st.n_r[tail_r0 + i] = g->hcnt[C_TAIL + 1 + i];
+            g->st.a_r[tail_r0 + i] = (int64_t)dense_entries(g->hcnt[C_TAIL + 1 + i]);
+        }
+        r = tail_r0 + (int)k;
+        g->st.rounds = r;
     }
     for (int rr = 0; rr < r; ++rr) {
         if (g->st.a_r[rr] >= 0) continue;
@@ -795,6 +819,8 @@ mst_status mst_set_option(mst_graph* g, int option, int64_t value) {
         if (value != 0 && value != 1) return fail(MST_EINVAL, "option value must be 0 or 1");
         if (option == MST_OPT_DENSE) {
             g->opt_dense = value != 0;
+        } else if (option == MST_OPT_DEVICE_TAIL) {
+            g->opt_tail = value != 0;
         } else if (option == MST_OPT_KEEP_EDGES) {
             if (value && !g->L && g->n > 0) {
                 CKS(galloc(g, &g->L, g->n));

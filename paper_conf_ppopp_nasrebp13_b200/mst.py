@@ -27,7 +27,7 @@ EXPORTS = ["mst_create", "mst_create_host", "mst_run", "mst_run_host", "mst_solv
            "mst_destroy", "mst_last_error", "mst_get_stats", "mst_set_profiling",
            "mst_get_unique_id", "mst_create_dist", "mst_create_sim", "mst_version",
            "mst_set_option"]
-MST_OPT_DENSE, MST_OPT_KEEP_EDGES = 1, 2
+MST_OPT_DENSE, MST_OPT_KEEP_EDGES, MST_OPT_DEVICE_TAIL = 1, 2, 3
 
 
 class mst_stats(ctypes.Structure):

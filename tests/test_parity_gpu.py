@@ -247,8 +247,12 @@ def test_options_switch_on_one_handle(lib, oracle_mod, gg):
             h.set_option(99, 1)
 
 
-@pytest.mark.parametrize("k,sd", [(1, 0), (4, 6), (5, 6)])
-def test_dense_rounds_used(lib, oracle_mod, gg, k, sd):
+@pytest.mark.parametrize("tail", [1, 0])
+@pytest.mark.parametrize("k,sd", [(1, 0), (4, 6), (5, 6), (3, 6), (2, 4)])
+def test_dense_rounds_used(lib, oracle_mod, gg, k, sd, tail):
+    """dense rounds both in the cooperative device tail and as per-round launches"""
     g = gg.config(k, s=3, scale_down=sd)
-    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w)
+    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, runs=2,
+                       options=[(lib.mst.MST_OPT_DEVICE_TAIL, tail)])
     assert st["dense_round"] >= 0
+    assert st["n_r"][-1] <= 1 or st["rounds"] >= 1
