@@ -23,6 +23,7 @@ cudaError_t launch_degree(cudaStream_t st, int nsm, u32 n, u32 m, const int* src
                           u32* eu, u32* ev, u32* deg, u32* err);
 cudaError_t launch_scan_rows(cudaStream_t st, u32 n, const u32* deg, u32* row, u32* cursor,
                              u64* status, u32 epoch);
+cudaError_t set_owner_policy(int p);
 cudaError_t launch_reorder(cudaStream_t st, int nsm, u32 n, u32 m, const u32* deg, u32* degn,
                            u32* eu, u32* ev, u32* newid, u32* counts, u64* status, u32 epoch,
                            u32* odeg);

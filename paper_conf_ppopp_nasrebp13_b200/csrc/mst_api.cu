@@ -293,7 +293,13 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CK(cudaStreamSynchronize(g->cst));
     if (g->hcnt[0]) return fail(MST_EINVAL, "an endpoint is outside [0, n) (n = %lld)", (long long)n);
 
-    // owner degrees (each non-loop edge once, owned by its lower internal endpoint)
+    // owner degrees (each non-loop edge once, owned by one endpoint: owner_of())
+    {
+        // default: the higher internal id (the lower-degree endpoint) owns the record, so
+        // the random per-record work lands on the hot hub labels; MST_OWNER_MAX=0 reverts
+        const char* op = getenv("MST_OWNER_MAX");
+        CK(set_owner_policy(op && op[0] == '0' ? 0 : 1));
+    }
     CK(cudaMemsetAsync(cursor, 0, std::max<u64>(n, 1) * sizeof(u32), g->cst));
     const char* ro = getenv("MST_REORDER");  // "0": keep the caller's vertex numbering
     if (n > 0 && reorder && !(ro && ro[0] == '0')) {
