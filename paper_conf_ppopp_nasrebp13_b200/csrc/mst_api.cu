@@ -395,7 +395,7 @@ mst_status create_common(int64_t n, int64_t m, const int32_t* src, const int32_t
         return fail(MST_ECUDA, "device setup: %s", cudaGetErrorString(e));
     }
     mst_status s = build(g, src, dst, (const unsigned*)w, nshards_sim, rank, nranks, reorder);
-    if (s == MST_OK && nranks > 1) {
+    if (s == MST_OK && id != nullptr) {  // mst_create_dist: NCCL communicator (also 1 rank)
         ncclUniqueId uid;
         memcpy(&uid, id, sizeof uid);
         ncclResult_t r = ncclCommInitRank(&g->comm, nranks, uid, rank);

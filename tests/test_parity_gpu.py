@@ -256,3 +256,25 @@ def test_dense_rounds_used(lib, oracle_mod, gg, k, sd, tail):
                        options=[(lib.mst.MST_OPT_DEVICE_TAIL, tail)])
     assert st["dense_round"] >= 0
     assert st["n_r"][-1] <= 1 or st["rounds"] >= 1
+
+
+# ------------------------------------------------------------------ distributed path, 1 rank
+@pytest.mark.parametrize("k,sd", [(1, 0), (4, 8), (3, 8), (5, 6)])
+def test_dist_single_rank_nccl(lib, oracle_mod, gg, k, sd):
+    """mst_create_dist with nranks = 1: a real NCCL communicator and the per-round
+    ncclAllReduce(MIN) of best (and of the min-matrix at the dense transition) on one GPU."""
+    g = gg.config(k, s=6, scale_down=sd)
+    try:
+        uid = lib.mst_get_unique_id()
+    except lib.MSTError as e:
+        pytest.skip(f"NCCL unique id unavailable: {e}")
+    o_ids, o_tot = oracle_mod.kruskal(g.n, g.src, g.dst, g.w)
+    with lib.MSTGraph(g.n, dev(g.src), dev(g.dst), dev(g.w), dist=(uid, 0, 1)) as h:
+        h.set_profiling(True)
+        for opts in ([], [(lib.mst.MST_OPT_DEVICE_TAIL, 0)], [(lib.mst.MST_OPT_KEEP_EDGES, 1)]):
+            for o, v in opts:
+                h.set_option(o, v)
+            ids, cnt, tot = h.run()
+            assert np.array_equal(ids.cpu().numpy(), o_ids) and tot == o_tot
+        st = h.stats()
+        assert st["nranks"] == 1 and st["kernel_launches"]["comm"] >= 1
