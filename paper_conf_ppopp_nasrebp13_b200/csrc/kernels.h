@@ -23,15 +23,15 @@ cudaError_t launch_degree(cudaStream_t st, int nsm, u32 n, u32 m, const int* src
                           u32* eu, u32* ev, u32* deg, u32* err);
 cudaError_t launch_scan_rows(cudaStream_t st, u32 n, const u32* deg, u32* row, u32* cursor,
                              u64* status, u32 epoch);
-cudaError_t set_owner_policy(int p);
 cudaError_t launch_reorder(cudaStream_t st, int nsm, u32 n, u32 m, const u32* deg, u32* degn,
                            u32* eu, u32* ev, u32* newid, u32* counts, u64* status, u32 epoch,
-                           u32* odeg);
+                           u32* odeg, int hi_owner);
 u64 reorder_scratch(u64 n);
 cudaError_t launch_owner_degree(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
-                                u32* odeg);
+                                u32* odeg, int hi_owner);
 cudaError_t launch_scatter(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
-                           const unsigned* w, u32* cursor, uint4* arcs, uint2* euv);
+                           const unsigned* w, u32* cursor, uint4* arcs, uint2* euv,
+                           int hi_owner);
 cudaError_t launch_min0(cudaStream_t st, int nsm, u64 A, const uint4* arcs, u64* best, u32 nb,
                         u32* tile_ctrs, u32 seq);
 cudaError_t launch_hook(cudaStream_t st, u32 nr, const u64* best, u64* best_next, u64* hmap, u32 tag,

@@ -141,15 +141,12 @@ struct mst_graph {
 
 namespace {
 
-bool g_pool_configured = false;
-
+// keep freed pool memory reserved for the next handle (per device, idempotent, thread-safe)
 mst_status configure_pool(int dev) {
-    if (g_pool_configured) return MST_OK;
     cudaMemPool_t pool;
     CK(cudaDeviceGetDefaultMemPool(&pool, dev));
     uint64_t thr = UINT64_MAX;
     CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
-    g_pool_configured = true;
     return MST_OK;
 }
 
@@ -294,12 +291,10 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     if (g->hcnt[0]) return fail(MST_EINVAL, "an endpoint is outside [0, n) (n = %lld)", (long long)n);
 
     // owner degrees (each non-loop edge once, owned by one endpoint: owner_of())
-    {
-        // default: the higher internal id (the lower-degree endpoint) owns the record, so
-        // the random per-record work lands on the hot hub labels; MST_OWNER_MAX=0 reverts
-        const char* op = getenv("MST_OWNER_MAX");
-        CK(set_owner_policy(op && op[0] == '0' ? 0 : 1));
-    }
+    // default: the higher internal id (the lower-degree endpoint) owns the record, so the
+    // random per-record work lands on the hot hub labels; MST_OWNER_MAX=0 reverts
+    const char* op = getenv("MST_OWNER_MAX");
+    const int hi_owner = (op && op[0] == '0') ? 0 : 1;
     CK(cudaMemsetAsync(cursor, 0, std::max<u64>(n, 1) * sizeof(u32), g->cst));
     const char* ro = getenv("MST_REORDER");  // "0": keep the caller's vertex numbering
     if (n > 0 && reorder && !(ro && ro[0] == '0')) {
@@ -310,9 +305,9 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
         CKS(galloc(g, &newid, n));
         CKS(galloc(g, &counts, reorder_scratch(n)));
         CK(launch_reorder(g->cst, g->nsm, (u32)n, (u32)m, deg, degn, g->eu, g->ev, newid, counts,
-                          g->status, g->epoch++, cursor));
+                          g->status, g->epoch++, cursor, hi_owner));
     } else {
-        CK(launch_owner_degree(g->cst, g->nsm, (u32)m, g->eu, g->ev, cursor));
+        CK(launch_owner_degree(g->cst, g->nsm, (u32)m, g->eu, g->ev, cursor, hi_owner));
     }
     deg = cursor;
     u32* odeg_scan_out;
@@ -329,7 +324,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     g->A0 = A0;
     CKS(galloc(g, &g->arcs0, A0));
     CKS(galloc(g, &g->euv, m));
-    CK(launch_scatter(g->cst, g->nsm, (u32)m, g->eu, g->ev, w, cursor, g->arcs0, g->euv));
+    CK(launch_scatter(g->cst, g->nsm, (u32)m, g->eu, g->ev, w, cursor, g->arcs0, g->euv, hi_owner));
 
     // shards: simulation = all G ranges locally; distributed = this rank's range only
     const int G = nshards_sim > 1 ? nshards_sim : nranks;
