@@ -129,9 +129,10 @@ def time_oracle(g, budget_s=30.0):
 def byte_model(st):
     """Algorithmic bytes per round.
 
-    sparse round r (A8): 16 B read per alive arc + 16 B written per surviving arc; the round
-    that switches to the dense matrix writes no arcs (its minima go to the L2-resident
-    matrix). dense round r (A9): 8 B per matrix entry read (n_r (n_r - 1) / 2 entries).
+    sparse round r (A8): 16 B read per edge record entering the pass + 16 B written per
+    surviving record when the pass compacts (MST_OPT_COMPACT_TAU: a pass whose records mostly
+    survive writes nothing; the next pass re-reads the same records); the round that switches
+    to the dense matrix writes no records (they go to the L2-resident matrix). dense round r (A9): 8 B per matrix entry read (n_r (n_r - 1) / 2 entries).
     The last round only hooks (<= 1 live component is left) and moves no arcs."""
     a, R, dr = st["a_r"], st["rounds"], st.get("dense_round", -1)
     out = []
@@ -143,7 +144,9 @@ def byte_model(st):
             out.append({"kind": "dense", "bytes": 8 * a[r]})
         else:
             nxt_sparse = not (dr >= 0 and r + 1 >= dr)
-            out.append({"kind": "filter", "bytes": 16 * a[r] + (16 * a[r + 1] if nxt_sparse else 0)})
+            comp = st.get("compacted", [True] * R)[r]
+            out.append({"kind": "filter", "compacted": bool(comp and nxt_sparse),
+                        "bytes": 16 * a[r] + (16 * a[r + 1] if (nxt_sparse and comp) else 0)})
     return out
 
 
@@ -178,6 +181,8 @@ def run_gpu(args):
         h.set_option(mstb.mst.MST_OPT_DENSE, 0)
     elif args.mode == "keep":
         h.set_option(mstb.mst.MST_OPT_KEEP_EDGES, 1)
+    if args.tau is not None:
+        h.set_option(mstb.mst.MST_OPT_COMPACT_TAU, args.tau)
     build_ms = h.stats()["build_ms"]
     out_ids = torch.empty(max(n - 1, 1), dtype=torch.int32, device="cuda")
     stream = torch.cuda.current_stream()
@@ -225,6 +230,8 @@ def run_gpu(args):
         filt_bytes += sum(x["bytes"] for x in bm if x["kind"] == "filter")
         if round_acc is None:
             round_acc = [{"r": r, "kind": bm[r]["kind"], "n_r": st["n_r"][r], "A_r": st["a_r"][r],
+                          "compacted": bm[r].get("compacted"),
+                          "survival_permille": st["survival_permille"][r],
                           "filter_ms": 0.0, "filter_bytes": bm[r]["bytes"]}
                          for r in range(st["rounds"])]
         for r in range(st["rounds"]):
@@ -365,6 +372,8 @@ def main():
     ap.add_argument("--mode", default="morph", choices=["morph", "sparse", "keep"],
                     help="morph: delete+compact, dense min-matrix at <= 4096 components "
                          "(default); sparse: never dense; keep: the paper's no-deletion scheme")
+    ap.add_argument("--tau", type=int, default=None,
+                    help="MST_OPT_COMPACT_TAU (permille; default: the library's)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-oracle", action="store_true")
     ap.add_argument("--ref-budget-s", type=float, default=150.0)

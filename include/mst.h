@@ -139,6 +139,11 @@ typedef struct {
     double round_filter_ms[MST_MAX_ROUNDS]; /* A8 (or A9 dense) kernel time per round     */
     int64_t gpu_launches;                 /* kernels launched by the last run            */
     int32_t dense_round;                  /* first round run on the dense min-matrix, -1 */
+    int64_t compacted_mask;               /* bit r: round r's pass compacted its records  */
+    int32_t survival_permille[MST_MAX_ROUNDS]; /* estimated survivors of pass r that its
+                                                  compaction decision used (-1: none)      */
+    int32_t hub_row;                      /* 1: the dense transition kept the top hub's
+                                             matrix row in shared memory (heavy tail)     */
 } mst_stats;
 
 mst_status mst_get_stats(const mst_graph* g, mst_stats* out);
@@ -160,8 +165,15 @@ mst_status mst_set_profiling(mst_graph* g, int enable);
  *       morph step (deletion) buys.
  *   MST_OPT_DEVICE_TAIL (default 1): once dense, run every remaining round inside one
  *       cooperative kernel (no host round trip per round); 0 = one launch set per round.
+ *   MST_OPT_COMPACT_TAU (default 950, permille in [0, 1000]): a sparse pass deletes the dead
+ *       edge records (compaction, the morph step) only when the sampled fraction of its
+ *       records that survive is below tau/1000; otherwise the next pass re-reads the same
+ *       records through the composed label map (row A7). 1000 = always compact, 0 = never
+ *       (deletion deferred to the dense transition). Decided on the device per pass from the
+ *       previous pass's exact survival (round 0: 4096 sampled records); never changes the
+ *       result.
  */
-enum { MST_OPT_DENSE = 1, MST_OPT_KEEP_EDGES = 2, MST_OPT_DEVICE_TAIL = 3 };
+enum { MST_OPT_DENSE = 1, MST_OPT_KEEP_EDGES = 2, MST_OPT_DEVICE_TAIL = 3, MST_OPT_COMPACT_TAU = 4 };
 mst_status mst_set_option(mst_graph* g, int option, int64_t value);
 
 /* ------------------------------------------------------------------ multi-GPU (§8(e))

@@ -6,7 +6,8 @@
 
 #define MST_CHAIN_MAX 64
 #define ACC_SLOTS 64  // forest weight/size accumulators: 64 (sum, count) pairs summed on the host
-#define DENSE_MAX 4096  // components: the dense min-matrix then holds <= 8.4 M entries (67 MB)
+#define DENSE_MAX 4096
+#define SAMPLES_PER_PASS 4096  // records sampled for a pass's compaction decision  // components: the dense min-matrix then holds <= 8.4 M entries (67 MB)
 
 namespace mstk {
 typedef uint32_t u32;
@@ -17,6 +18,22 @@ typedef uint64_t u64;
 struct MapChain {
     const int* m[MST_CHAIN_MAX];
     int len;
+};
+
+// Compaction decision of a sparse pass (MST_OPT_COMPACT_TAU): the pass deletes its dead
+// records only if the estimated surviving fraction num/den is below tau/1000, where (num,
+// den) is the previous pass's exact count or, for round 0, a sample. num == nullptr: the
+// host decided (compact unless `out` is null). Every pass counts its survivors into *surv and
+// its records into *seen (the next pass's estimate); block 0 writes the decision to *hword
+// (mapped host memory, tagged) for the host's bookkeeping at the next round.
+struct CompactCtl {
+    const u32* num = nullptr;
+    const u32* den = nullptr;
+    u32 tau = 1000;
+    u32* surv = nullptr;
+    u32* seen = nullptr;
+    u64* hword = nullptr;
+    u32 tag = 0;
 };
 
 cudaError_t launch_degree(cudaStream_t st, int nsm, u32 n, u32 m, const int* src, const int* dst,
@@ -38,11 +55,13 @@ cudaError_t launch_hook(cudaStream_t st, u32 nr, const u64* best, u64* best_next
                         const uint2* euv, const MapChain& chain, u32* P, int* Mtmp, u32* msf,
                         u64* acc, u64* status, u32 epoch, u32* n_next);
 cudaError_t launch_jump(cudaStream_t st, int nsm, u32 nr, u32* P, const int* Mtmp, int* Mr,
-                        const u32* nn, u64* best_next);
+                        const u32* nn, u64* best_next, const int* hub, int* hub_next);
 cudaError_t launch_filter_min(cudaStream_t st, int nsm, const u32* a_in, u64 a_max,
                               const uint4* in, const int* M, uint4* out, u64* best, u32 nb,
                               u64* status, u32 epoch, u32* a_next, u32* tile_ctrs, u32 seq,
-                              u64* mat);
+                              u64* mat, const CompactCtl& cc = CompactCtl(),
+                              const int* hub = nullptr);
+cudaError_t launch_dense_best(cudaStream_t st, int nsm, u32 n, const u64* mat, u64* best);
 cudaError_t launch_dense_init(cudaStream_t st, int nsm, u32 n, u64* mat);
 cudaError_t launch_dense_round(cudaStream_t st, int nsm, u32 n, const u64* mat, const int* M,
                                u32 n_next, u64* mat_next, u64* best_next);
@@ -50,7 +69,9 @@ u64 dense_entries(u64 n);
 cudaError_t launch_dense_tail(cudaStream_t st, int nsm, u32 n0, u64* best0, u64* best1,
                               u64* mat0, u64* mat1, const uint2* euv, const MapChain& chain,
                               u32* msf, u64* acc, u32* bar, u32* stats);
-cudaError_t launch_label_update(cudaStream_t st, int nsm, u32 n, int* L, const int* Mr, bool first);
+cudaError_t launch_compose(cudaStream_t st, int nsm, u32 nb, const int* src, const int* Mr, int* phi);
+cudaError_t launch_sample_survival(cudaStream_t st, const uint4* in, const u32* a_ptr, const int* M,
+                                   u32* num, u32* den);
 cudaError_t launch_output(cudaStream_t st, u32 nwords, const u32* msf, int* out, u64* status,
                           u32 epoch, u32* out_count);
 cudaError_t launch_combine_min(cudaStream_t st, int nsm, u32 nr, int nshards, u64* shard_best,

@@ -79,7 +79,12 @@ constexpr int AREC_STRIDE = MST_MAX_ROUNDS + 1;
 inline int arec(int j, int r) { return C_AREC + j * AREC_STRIDE + r; }
 constexpr int C_BAR = C_AREC + 64 * AREC_STRIDE;  // grid barrier {count, generation}
 constexpr int C_TAIL = C_BAR + 2;                   // device tail: rounds, n per round
-constexpr int DCNT_WORDS = C_TAIL + 1 + MST_MAX_ROUNDS;
+constexpr int C_SEEN = C_TAIL + 1 + MST_MAX_ROUNDS;  // records entering pass r (all shards)
+constexpr int C_SURV = C_SEEN + MST_MAX_ROUNDS;       // survivors of pass r (all shards)
+constexpr int C_SAMP = C_SURV + MST_MAX_ROUNDS;       // round-0 sample: {alive, samples}
+constexpr int C_HUB = C_SAMP + 2;  // label of internal vertex 0 (the top hub) per round
+constexpr int DCNT_WORDS = C_HUB + MST_MAX_ROUNDS + 1;
+constexpr int HSURV = MST_MAX_ROUNDS + 1;  // mapped words: [0, HSURV) sizes, [HSURV, 2 HSURV) decisions
 
 struct Shard {
     u64 lo, hi;  // arc range [lo, hi) in arcs_0 and in the ping-pong buffers
@@ -115,7 +120,8 @@ struct mst_graph {
     u32* dcnt = nullptr;
     u64* acc = nullptr;
     u32* hcnt = nullptr;  // pinned
-    volatile u64* hmap = nullptr;  // pinned + mapped: tagged n_{r+1} written by the hook
+    volatile u64* hmap = nullptr;  // pinned + mapped: tagged n_{r+1} written by the hook,
+                                   // then (at HSURV + r) the sampled compaction decision
     u64* dmap = nullptr;           // its device alias
     u32 run_seq = 0;
     u64* hacc = nullptr;  // pinned
@@ -129,7 +135,9 @@ struct mst_graph {
     bool opt_dense = true;   // MST_OPT_DENSE
     bool opt_keep = false;   // MST_OPT_KEEP_EDGES (paper-faithful ablation)
     bool opt_tail = true;    // MST_OPT_DEVICE_TAIL
-    int* L = nullptr;        // vertex -> component labels (keep-edges mode, row A7)
+    u32 tau = 950;           // MST_OPT_COMPACT_TAU (permille)
+    bool hub_row = false;    // heavy-tailed input: hub row of the dense transition in smem
+    int* phi = nullptr;      // composed label map of the records' label space (row A7)
 
     bool prof = false;
     std::vector<ProfRec> recs;
@@ -279,8 +287,8 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CK(cudaMallocHost(&g->hacc, 2 * ACC_SLOTS * sizeof(u64)));
     {
         void* hm = nullptr;
-        CK(cudaHostAlloc(&hm, (MST_MAX_ROUNDS + 1) * sizeof(u64), cudaHostAllocMapped));
-        memset(hm, 0, (MST_MAX_ROUNDS + 1) * sizeof(u64));
+        CK(cudaHostAlloc(&hm, 2 * HSURV * sizeof(u64), cudaHostAllocMapped));
+        memset(hm, 0, 2 * HSURV * sizeof(u64));
         g->hmap = (volatile u64*)hm;
         CK(cudaHostGetDevicePointer((void**)&g->dmap, hm, 0));
     }
@@ -306,6 +314,12 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
         CKS(galloc(g, &counts, reorder_scratch(n)));
         CK(launch_reorder(g->cst, g->nsm, (u32)n, (u32)m, deg, degn, g->eu, g->ev, newid, counts,
                           g->status, g->epoch++, cursor, hi_owner));
+        // heavy-tailed degrees (internal vertex 0 = the top hub far above the mean degree):
+        // the dense transition then keeps the hub's matrix row in shared memory
+        u32 d0 = 0;
+        CK(cudaMemcpyAsync(&d0, degn, sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
+        CK(cudaStreamSynchronize(g->cst));
+        g->hub_row = (double)d0 * (double)n >= 16.0 * 2.0 * (double)m;
     } else {
         CK(launch_owner_degree(g->cst, g->nsm, (u32)m, g->eu, g->ev, cursor, hi_owner));
     }
@@ -346,6 +360,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CKS(galloc(g, &g->Mtmp, n));
     CKS(galloc(g, &g->maps, 2 * n + 1));  // sum_r n_r <= 2n: every live component merges
     CKS(galloc(g, &g->msf, g->nwords));
+    CKS(galloc(g, &g->phi, n));
     if (n >= 2) {  // dense min-matrices (A9 / NEXT-1), <= 67 MB each
         CKS(galloc(g, &g->mat[0], dense_entries(n)));
         CKS(galloc(g, &g->mat[1], dense_entries(n)));
@@ -410,30 +425,41 @@ mst_status create_common(int64_t n, int64_t m, const int32_t* src, const int32_t
 // --------------------------------------------------------------------------- run
 // Spin on the tagged word the hook writes to mapped host memory (no memcpy, no stream sync);
 // a failing kernel never writes it, so the stream is queried now and then for errors.
-mst_status wait_round(mst_graph* g, cudaStream_t s, int r, u32 tag, u32* nn) {
+mst_status wait_word(mst_graph* g, cudaStream_t s, int idx, u32 tag, u32* val) {
     const auto t0 = std::chrono::steady_clock::now();
     for (u64 spin = 0;; ++spin) {
-        const u64 v = g->hmap[r];
+        const u64 v = g->hmap[idx];
         if ((u32)(v >> 32) == tag) {
-            *nn = (u32)v;
+            *val = (u32)v;
             return MST_OK;
         }
         if ((spin & 1023) == 1023) {
             const cudaError_t e = cudaStreamQuery(s);
             if (e != cudaSuccess && e != cudaErrorNotReady)
-                return fail(MST_ECUDA, "round %d: %s", r, cudaGetErrorString(e));
+                return fail(MST_ECUDA, "word %d: %s", idx, cudaGetErrorString(e));
             if (e == cudaSuccess) {  // stream drained: the word must be visible now
-                const u64 w = g->hmap[r];
+                const u64 w = g->hmap[idx];
                 if ((u32)(w >> 32) == tag) {
-                    *nn = (u32)w;
+                    *val = (u32)w;
                     return MST_OK;
                 }
-                return fail(MST_EINTERNAL, "round %d: size word not written", r);
+                return fail(MST_EINTERNAL, "word %d: not written", idx);
             }
             if (std::chrono::steady_clock::now() - t0 > std::chrono::seconds(120))
-                return fail(MST_EINTERNAL, "round %d: timed out waiting for the hook", r);
+                return fail(MST_EINTERNAL, "word %d: timed out waiting for the device", idx);
         }
     }
+}
+// Spin on the tagged word the hook writes to mapped host memory (no memcpy, no stream sync);
+// a failing kernel never writes it, so the stream is queried now and then for errors.
+mst_status wait_round(mst_graph* g, cudaStream_t s, int r, u32 tag, u32* nn) {
+    return wait_word(g, s, r, tag, nn);
+}
+
+bool use_hub_row(const mst_graph* g) {
+    static const char* e = getenv("MST_HUB_ROW");  // "0" / "1": override (ablation)
+    if (e && (e[0] == '0' || e[0] == '1')) return e[0] == '1';
+    return g->hub_row;
 }
 
 mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out_num,
@@ -466,6 +492,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         CK(cudaMemsetAsync(g->msf, 0, std::max<u64>(g->nwords, 1) * sizeof(u32), s));
         CK(cudaMemsetAsync(g->acc, 0, 2 * ACC_SLOTS * sizeof(u64), s));
         if (g->sim) CK(cudaMemsetAsync(g->shard_best, 0xff, n * G * sizeof(u64), s));
+        CK(cudaMemsetAsync(g->dcnt + C_SEEN, 0, 2 * MST_MAX_ROUNDS * sizeof(u32), s));
+        CK(cudaMemsetAsync(g->dcnt + C_HUB, 0, sizeof(u32), s));  // round 0: vertex 0 itself
     }
     // ---- A2 round-0 minimum (+ A3)
     for (int j = 0; j < G; ++j) {
@@ -497,7 +525,28 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     u32 nr = (u32)n;
     u64* bcur = g->bestA;
     u64* bnxt = g->bestB;
-    int r = 0, outb = 0;
+    int r = 0;
+    // where the alive records live: buffer `cur` (per-shard windows), labels of round `brnd`
+    // (n_b = nb_sz labels); a pass whose compaction was decided on the device (sampled) is
+    // resolved at the next round's wait (pend)
+    const uint4* cur = g->arcs0;
+    int brnd = 0;
+    u32 nb_sz = (u32)n;
+    int pend = -1;
+    const uint4* pend_out = nullptr;
+    g->st.compacted_mask = 0;
+    g->st.hub_row = 0;
+    for (int i = 0; i < MST_MAX_ROUNDS; ++i) g->st.survival_permille[i] = -1;
+    auto resolve = [&](u32 word) {  // outcome of round pend's sampled decision
+        g->st.survival_permille[pend] = (int32_t)(word >> 1);  // the estimate the pass used
+        if (word & 1u) {
+            cur = pend_out;
+            brnd = pend + 1;
+            nb_sz = (u32)g->st.n_r[pend + 1];
+            g->st.compacted_mask |= 1ll << pend;
+        }
+        pend = -1;
+    };
     bool dense = false;  // this round's alive arcs live in the min-matrix g->mat[mc]
     int mc = 0;
     g->st.dense_round = -1;
@@ -522,7 +571,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         {   // the jump does not need the host: it reads n_{r+1} on the device and runs
             // while the counts travel to the host
             Prof p(g, s, MST_K_JUMP, r);
-            CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, Mr, g->dcnt + C_NNEXT, bnxt));
+            CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, Mr, g->dcnt + C_NNEXT, bnxt,
+                           (const int*)g->dcnt + C_HUB + r, (int*)g->dcnt + C_HUB + r + 1));
         }
         // one host round trip per round: n_{r+1} (sizes round r's filter),
         // read zero-copy from the word the hook's last tile writes to mapped host memory
@@ -530,6 +580,11 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         CKS(wait_round(g, s, r, tag_base | (u32)r, &nn));
         g->st.n_r[r] = nr;
         g->st.a_r[r] = dense ? (int64_t)dense_entries(nr) : -1;  // sparse: filled at the end
+        if (pend >= 0) {  // the previous pass decided on the device whether it compacted
+            u32 word;
+            CKS(wait_word(g, s, HSURV + pend, tag_base | (u32)pend, &word));
+            resolve(word);
+        }
         if (nn <= 1) {  // <= 1 live component left: no inter-component edge remains
             ++r;
             break;
@@ -544,42 +599,87 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         } else {
             to_dense = g->mat[0] && g->opt_dense && !g->opt_keep && nn <= (u32)DENSE_MAX;
             if (to_dense) CK(launch_dense_init(s, g->nsm, nn, g->mat[0]));
-            if (g->opt_keep) {  // A7: the vertex -> component map, explicitly
+            // A7: the map of this round's pass, from the records' label space (round brnd)
+            // to round r+1: M_r itself, or composed over the rounds that did not compact
+            const int* Mpass = Mr;
+            if (brnd < r) {
                 Prof p(g, s, MST_K_JUMP, r);
-                CK(launch_label_update(s, g->nsm, (u32)n, g->L, Mr, r == 0));
+                const int* src = (brnd == r - 1) ? chain.m[chain.len - 1] : g->phi;
+                CK(launch_compose(s, g->nsm, nb_sz, src, Mr, g->phi));
+                Mpass = g->phi;
+            }
+            // compaction policy: never (keep-edges: the paper's scheme, or tau = 0), always
+            // (tau >= 1000), or decided on the device from the estimated survival (CompactCtl)
+            const bool never = g->opt_keep || g->tau == 0;
+            int dsh = -1;  // the shard whose pass reports the device-side decision
+            for (int j = 0; j < G && dsh < 0; ++j)
+                if (g->shards[j].hi > g->shards[j].lo) dsh = j;
+            const bool adaptive = !to_dense && !never && g->tau < 1000 && dsh >= 0;
+            const uint4* outbuf = (cur == g->abuf[0]) ? g->abuf[1] : g->abuf[0];
+            CompactCtl cc;
+            cc.surv = g->dcnt + C_SURV + r;
+            cc.seen = g->dcnt + C_SEEN + r;
+            if (adaptive) {
+                cc.tau = g->tau;
+                if (r == 0) {  // no previous pass: sample this pass's records
+                    Prof p(g, s, MST_K_JUMP, r);
+                    const Shard& sh = g->shards[dsh];
+                    CK(launch_sample_survival(s, cur + sh.lo, g->dcnt + arec(dsh, r), Mpass,
+                                              g->dcnt + C_SAMP, g->dcnt + C_SAMP + 1));
+                    cc.num = g->dcnt + C_SAMP;
+                    cc.den = g->dcnt + C_SAMP + 1;
+                } else {
+                    cc.num = g->dcnt + C_SURV + (r - 1);
+                    cc.den = g->dcnt + C_SEEN + (r - 1);
+                }
             }
             for (int j = 0; j < G; ++j) {
                 Shard& sh = g->shards[j];
                 u64* tgt = g->sim ? g->shard_best + (u64)j * n : bnxt;
                 Prof p(g, s, MST_K_FILTER, r);
-                if (g->opt_keep) {
-                    // the paper's scheme: every original record, every round
-                    const u64 A0j = sh.hi - sh.lo;
-                    CK(launch_filter_min(s, g->nsm, nullptr, A0j, g->arcs0 + sh.lo, g->L, nullptr,
-                                         tgt, nn, g->status, g->epoch++, g->dcnt + arec(j, r + 1),
-                                         g->dcnt + C_TILE, g->pass_seq++, nullptr));
-                    continue;
+                uint4* out = (never || to_dense) ? nullptr : const_cast<uint4*>(outbuf) + sh.lo;
+                CompactCtl ccj = cc;
+                if (adaptive && j == dsh) {
+                    ccj.hword = g->dmap + HSURV + r;
+                    ccj.tag = tag_base | (u32)r;
                 }
-                const uint4* in = (r == 0 ? g->arcs0 : g->abuf[outb ^ 1]) + sh.lo;
-                CK(launch_filter_min(s, g->nsm, g->dcnt + arec(j, r), sh.A, in, Mr,
-                                     g->abuf[outb] + sh.lo, tgt, nn, g->status, g->epoch++,
+                CK(launch_filter_min(s, g->nsm, g->dcnt + arec(j, r), sh.hi - sh.lo, cur + sh.lo,
+                                     Mpass, out, tgt, nn, g->status, g->epoch++,
                                      g->dcnt + arec(j, r + 1), g->dcnt + C_TILE, g->pass_seq++,
-                                     to_dense ? g->mat[0] : nullptr));
+                                     to_dense ? g->mat[0] : nullptr, ccj,
+                                     (to_dense && use_hub_row(g))
+                                         ? (const int*)g->dcnt + C_HUB + r + 1 : nullptr));
+            }
+            if (to_dense && use_hub_row(g)) g->st.hub_row = 1;
+            if (adaptive) {
+                pend = r;
+                pend_out = outbuf;
+            } else if (!never && !to_dense) {
+                cur = outbuf;
+                brnd = r + 1;
+                nb_sz = nn;
+                g->st.compacted_mask |= 1ll << r;
             }
         }
         chain.m[chain.len++] = Mr;
         moff += nr;
         ++r;
-        outb ^= 1;
-        if (g->sim && !dense) {
+        if (to_dense) {
+            // the transition pass filled only the matrix: every rank needs all of it for the
+            // replicated dense rounds, and the first dense round's minima come from it
+            if (g->comm) {
+                Prof p(g, s, MST_K_COMM, r);
+                CKN(ncclAllReduce(g->mat[0], g->mat[0], dense_entries(nn), ncclUint64, ncclMin,
+                                  g->comm, s));
+            }
+            Prof p(g, s, MST_K_DENSE, r);
+            CK(launch_dense_best(s, g->nsm, nn, g->mat[0], bnxt));
+        } else if (g->sim && !dense) {
             Prof p(g, s, MST_K_COMM, r);
             CK(launch_combine_min(s, g->nsm, nn, G, g->shard_best, n, bnxt));
         } else if (g->comm && !dense) {
             Prof p(g, s, MST_K_COMM, r);
             CKN(ncclAllReduce(bnxt, bnxt, nn, ncclUint64, ncclMin, g->comm, s));
-            if (to_dense)  // every rank needs the full matrix for the replicated dense rounds
-                CKN(ncclAllReduce(g->mat[0], g->mat[0], dense_entries(nn), ncclUint64, ncclMin,
-                                  g->comm, s));
         }
         if (to_dense) {
             dense = true;
@@ -611,6 +711,11 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     CK(cudaMemcpyAsync(g->hcnt, g->dcnt, 2 * sizeof(u32), cudaMemcpyDeviceToHost, s));
     CK(cudaMemcpyAsync(g->hacc, g->acc, 2 * ACC_SLOTS * sizeof(u64), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
+    if (pend >= 0) {  // the last sampled decision (stats only)
+        u32 word;
+        CKS(wait_word(g, s, HSURV + pend, tag_base | (u32)pend, &word));
+        resolve(word);
+    }
     for (int i = 1; i < ACC_SLOTS; ++i) {  // sum the spread accumulators
         g->hacc[0] += g->hacc[2 * i];
         g->hacc[1] += g->hacc[2 * i + 1];
@@ -817,16 +922,18 @@ mst_status mst_get_stats(const mst_graph* g, mst_stats* out) {
 mst_status mst_set_option(mst_graph* g, int option, int64_t value) {
     return guarded([&]() -> mst_status {
         if (!g) return fail(MST_EINVAL, "handle is NULL");
+        if (option == MST_OPT_COMPACT_TAU) {
+            if (value < 0 || value > 1000)
+                return fail(MST_EINVAL, "MST_OPT_COMPACT_TAU must be in [0, 1000] (permille)");
+            g->tau = (u32)value;
+            return MST_OK;
+        }
         if (value != 0 && value != 1) return fail(MST_EINVAL, "option value must be 0 or 1");
         if (option == MST_OPT_DENSE) {
             g->opt_dense = value != 0;
         } else if (option == MST_OPT_DEVICE_TAIL) {
             g->opt_tail = value != 0;
         } else if (option == MST_OPT_KEEP_EDGES) {
-            if (value && !g->L && g->n > 0) {
-                CKS(galloc(g, &g->L, g->n));
-                CK(cudaStreamSynchronize(g->cst));
-            }
             g->opt_keep = value != 0;
         } else {
             return fail(MST_EINVAL, "unknown option %d", option);

@@ -27,7 +27,7 @@ EXPORTS = ["mst_create", "mst_create_host", "mst_run", "mst_run_host", "mst_solv
            "mst_destroy", "mst_last_error", "mst_get_stats", "mst_set_profiling",
            "mst_get_unique_id", "mst_create_dist", "mst_create_sim", "mst_version",
            "mst_set_option"]
-MST_OPT_DENSE, MST_OPT_KEEP_EDGES, MST_OPT_DEVICE_TAIL = 1, 2, 3
+MST_OPT_DENSE, MST_OPT_KEEP_EDGES, MST_OPT_DEVICE_TAIL, MST_OPT_COMPACT_TAU = 1, 2, 3, 4
 
 
 class mst_stats(ctypes.Structure):
@@ -42,6 +42,9 @@ class mst_stats(ctypes.Structure):
         ("round_filter_ms", ctypes.c_double * MAX_ROUNDS),
         ("gpu_launches", ctypes.c_int64),
         ("dense_round", ctypes.c_int32),
+        ("compacted_mask", ctypes.c_int64),
+        ("survival_permille", ctypes.c_int32 * MAX_ROUNDS),
+        ("hub_row", ctypes.c_int32),
     ]
 
 
@@ -181,7 +184,7 @@ class MSTGraph:
         return out[: cnt.value], int(cnt.value), int(tot.value)
 
     def set_option(self, option: int, value: int):
-        """mst_set_option: MST_OPT_DENSE / MST_OPT_KEEP_EDGES (include/mst.h)."""
+        """mst_set_option: MST_OPT_DENSE / _KEEP_EDGES / _DEVICE_TAIL / _COMPACT_TAU (include/mst.h)."""
         _check(load().mst_set_option(self._h, int(option), int(value)))
 
     def set_profiling(self, on: bool):
@@ -202,6 +205,9 @@ class MSTGraph:
             "round_filter_ms": list(s.round_filter_ms[:R]),
             "gpu_launches": s.gpu_launches,
             "dense_round": s.dense_round,
+            "compacted": [bool((s.compacted_mask >> r) & 1) for r in range(R)],
+            "survival_permille": list(s.survival_permille[:R]),
+            "hub_row": bool(s.hub_row),
         }
 
     def debug_filter_pass(self, map_kind=0, group=1, iters=5, stream=None):

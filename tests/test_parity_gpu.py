@@ -124,6 +124,28 @@ def test_star_huge_degree(lib, oracle_mod):
     assert_parity(lib, oracle_mod, n, src, dst, w)
 
 
+@pytest.mark.parametrize("seed", [0, 1])
+def test_hub_row_dense_transition(lib, oracle_mod, seed):
+    """a hub joined to every vertex by heavy edges, plus light random edges: many components
+    keep pairs with the hub's component until the dense transition, which reduces the hub's
+    matrix row in shared memory (heavy-tailed degrees switch it on)"""
+    rng = np.random.default_rng(seed)
+    n = 120_000
+    light = 150_000
+    s1 = rng.integers(1, n, light).astype(np.int32)
+    d1 = rng.integers(1, n, light).astype(np.int32)
+    w1 = rng.integers(0, 500, light).astype(np.uint32)
+    s2 = np.zeros(n - 1, np.int32)
+    d2 = np.arange(1, n, dtype=np.int32)
+    w2 = rng.integers(500, 1000, n - 1).astype(np.uint32)
+    for parts in ((s1, s2), (s2, s1)):  # hub edges last / first in id order
+        src = np.concatenate(parts)
+        dst = np.concatenate((d1, d2) if parts[0] is s1 else (d2, d1))
+        w = np.concatenate((w1, w2) if parts[0] is s1 else (w2, w1))
+        st = assert_parity(lib, oracle_mod, n, src, dst, w, runs=2)
+        assert st["dense_round"] >= 0 and st["hub_row"]
+
+
 def test_all_equal_weights(lib, oracle_mod, gg):
     g = gg.uniform(200_000, 800_000, 1, 2, 3, wlo=7, wmod=1)
     assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w)
@@ -232,6 +254,50 @@ def test_keep_edges_paper_scheme(lib, oracle_mod, gg, k, sd):
                        options=[(lib.mst.MST_OPT_KEEP_EDGES, 1)], runs=2)
     assert st["dense_round"] == -1
     assert all(a == st["arcs0"] for a in st["a_r"])  # nothing is ever deleted
+
+
+@pytest.mark.parametrize("tau", [0, 300, 900, 1000])
+@pytest.mark.parametrize("k,sd", [(1, 0), (2, 6), (3, 8), (4, 8), (5, 6)])
+def test_compaction_policy(lib, oracle_mod, gg, k, sd, tau):
+    """MST_OPT_COMPACT_TAU: a pass compacts only when its sampled survival is below tau;
+    otherwise later passes re-read the same records through the composed label map (row A7).
+    Every policy -- never (0), adaptive, always (1000) -- gives the identical forest, also
+    with the dense rounds off (long chains of non-compacting sparse passes)."""
+    g = gg.config(k, s=7, scale_down=sd)
+    for extra in ([], [(lib.mst.MST_OPT_DENSE, 0)]):
+        st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, runs=2,
+                           options=[(lib.mst.MST_OPT_COMPACT_TAU, tau)] + extra)
+        sparse = [r for r in range(st["rounds"] - 1)
+                  if st["dense_round"] < 0 or r + 1 < st["dense_round"]]
+        if tau == 0:
+            assert not any(st["compacted"])
+        if tau == 1000:
+            assert all(st["compacted"][r] for r in sparse)
+        for r in range(1, st["rounds"]):  # a non-compacting pass keeps every record
+            if r - 1 in sparse and r in sparse and not st["compacted"][r - 1]:
+                assert st["a_r"][r] == st["a_r"][r - 1]
+        for r in sparse:
+            sp = st["survival_permille"][r]
+            if 0 < tau < 1000:
+                assert 0 <= sp <= 1000 and st["compacted"][r] == (sp < tau)
+            else:
+                assert sp == -1
+
+
+def test_compaction_policy_sharded(lib, oracle_mod, gg):
+    """the sampled decision is taken once per pass for every shard of a simulated split"""
+    g = gg.config(4, s=8, scale_down=8)
+    for tau in (0, 700, 1000):
+        assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, nshards=3, runs=2,
+                      options=[(lib.mst.MST_OPT_COMPACT_TAU, tau), (lib.mst.MST_OPT_DENSE, 0)])
+
+
+def test_compaction_tau_range(lib, gg):
+    g = gg.config(1)
+    with lib.MSTGraph(g.n, dev(g.src), dev(g.dst), dev(g.w)) as h:
+        for bad in (-1, 1001):
+            with pytest.raises(lib.MSTError):
+                h.set_option(lib.mst.MST_OPT_COMPACT_TAU, bad)
 
 
 def test_options_switch_on_one_handle(lib, oracle_mod, gg):
