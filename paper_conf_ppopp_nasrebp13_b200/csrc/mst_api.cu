@@ -136,7 +136,8 @@ struct mst_graph {
     bool opt_keep = false;   // MST_OPT_KEEP_EDGES (paper-faithful ablation)
     bool opt_tail = true;    // MST_OPT_DEVICE_TAIL
     u32 tau = 950;           // MST_OPT_COMPACT_TAU (permille)
-    bool hub_row = false;    // heavy-tailed input: hub row of the dense transition in smem
+    bool hub_row = false;
+    u64* trace = nullptr;    // MST_TAIL_TRACE=1 (tools): phase timestamps of the dense tail    // heavy-tailed input: hub row of the dense transition in smem
     int* phi = nullptr;      // composed label map of the records' label space (row A7)
 
     bool prof = false;
@@ -184,6 +185,7 @@ void release(mst_graph* g) {
     if (g->hcnt) cudaFreeHost(g->hcnt);
     if (g->hacc) cudaFreeHost(g->hacc);
     if (g->hmap) cudaFreeHost((void*)g->hmap);
+    if (g->trace) cudaFree(g->trace);
     for (auto e : g->evpool) cudaEventDestroy(e);
     if (g->cst) cudaStreamDestroy(g->cst);
     delete g;
@@ -557,8 +559,26 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         if (dense && g->opt_tail) {
             // every remaining round in one cooperative launch (A4/A5/A6/A9 on the device)
             Prof p(g, s, MST_K_DENSE, r);
+            static const bool tr = getenv("MST_TAIL_TRACE") && getenv("MST_TAIL_TRACE")[0] == '1';
+            if (tr && !g->trace) {
+                CK(cudaMalloc(&g->trace, 64 * sizeof(u64)));
+                CK(cudaMemsetAsync(g->trace, 0, 64 * sizeof(u64), s));
+            }
             CK(launch_dense_tail(s, g->nsm, nr, bcur, bnxt, g->mat[mc], g->mat[mc ^ 1], g->euv,
-                                 chain, g->msf, g->acc, g->dcnt + C_BAR, g->dcnt + C_TAIL));
+                                 chain, g->msf, g->acc, g->dcnt + C_BAR, g->dcnt + C_TAIL,
+                                 tr ? g->trace : nullptr));
+            if (tr) {
+                u64 h[64];
+                CK(cudaMemcpyAsync(h, g->trace, sizeof h, cudaMemcpyDeviceToHost, s));
+                CK(cudaStreamSynchronize(s));
+                for (int k = 0; k < 8 && h[k * 8]; ++k) {
+                    fprintf(stderr, "tail round %d:", k);
+                    for (int q = 1; q < 8; ++q)
+                        fprintf(stderr, " %+.1f", h[k * 8 + q] ? (double)(h[k * 8 + q] - h[k * 8]) / 1e3 : -1.0);
+                    fprintf(stderr, " us\n");
+                }
+                CK(cudaMemsetAsync(g->trace, 0, 64 * sizeof(u64), s));
+            }
             tail_r0 = r;
             break;
         }
