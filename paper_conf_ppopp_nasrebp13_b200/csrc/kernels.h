@@ -53,9 +53,11 @@ cudaError_t launch_min0(cudaStream_t st, int nsm, u64 A, const uint4* arcs, u64*
                         u32* tile_ctrs, u32 seq);
 cudaError_t launch_hook(cudaStream_t st, u32 nr, const u64* best, u64* best_next, u64* hmap, u32 tag,
                         const uint2* euv, const MapChain& chain, u32* P, int* Mtmp, u32* msf,
-                        u64* acc, u64* status, u32 epoch, u32* n_next);
-cudaError_t launch_jump(cudaStream_t st, int nsm, u32 nr, u32* P, const int* Mtmp, int* Mr,
-                        const u32* nn, u64* best_next, const int* hub, int* hub_next);
+                        u64* acc, u32* tcnt, u32* n_next);
+// tcnt: 2 * hook_tiles(n) words (tile counts, then their exclusive scan)
+cudaError_t launch_jump(cudaStream_t st, int nsm, u32 nr, u32* P, const int* Mtmp, const u32* tcnt,
+                        int* Mr, const u32* nn, u64* best_next, const int* hub, int* hub_next);
+u64 hook_tiles(u64 n);
 cudaError_t launch_filter_min(cudaStream_t st, int nsm, const u32* a_in, u64 a_max,
                               const uint4* in, const int* M, uint4* out, u64* best, u32 nb,
                               u64* status, u32 epoch, u32* a_next, u32* tile_ctrs, u32 seq,

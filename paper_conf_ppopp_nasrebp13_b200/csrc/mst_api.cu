@@ -112,6 +112,7 @@ struct mst_graph {
     u64 *bestA = nullptr, *bestB = nullptr, *shard_best = nullptr;
     u32* P = nullptr;
     int *Mtmp = nullptr, *maps = nullptr;
+    u32* tcnt = nullptr;  // hook tile counts and their scan (renumber offsets)
     u32* msf = nullptr;
     u64* mat[2] = {nullptr, nullptr};  // dense min-matrices over component pairs
     u64* status = nullptr;
@@ -360,6 +361,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     if (g->sim) CKS(galloc(g, &g->shard_best, n * (u64)g->shards.size()));
     CKS(galloc(g, &g->P, n));
     CKS(galloc(g, &g->Mtmp, n));
+    CKS(galloc(g, &g->tcnt, 2 * hook_tiles(n) + 2));
     CKS(galloc(g, &g->maps, 2 * n + 1));  // sum_r n_r <= 2n: every live component merges
     CKS(galloc(g, &g->msf, g->nwords));
     CKS(galloc(g, &g->phi, n));
@@ -585,13 +587,13 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         int* Mr = g->maps + moff;
         {
             Prof p(g, s, MST_K_HOOK, r);
-            CK(launch_hook(s, nr, bcur, bnxt, g->dmap + r, tag_base | (u32)r, g->euv, chain, g->P, g->Mtmp, g->msf, g->acc,
-                           g->status, g->epoch++, g->dcnt + C_NNEXT));
+            CK(launch_hook(s, nr, bcur, bnxt, g->dmap + r, tag_base | (u32)r, g->euv, chain, g->P,
+                           g->Mtmp, g->msf, g->acc, g->tcnt, g->dcnt + C_NNEXT));
         }
         {   // the jump does not need the host: it reads n_{r+1} on the device and runs
             // while the counts travel to the host
             Prof p(g, s, MST_K_JUMP, r);
-            CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, Mr, g->dcnt + C_NNEXT, bnxt,
+            CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, g->tcnt, Mr, g->dcnt + C_NNEXT, bnxt,
                            (const int*)g->dcnt + C_HUB + r, (int*)g->dcnt + C_HUB + r + 1));
         }
         // one host round trip per round: n_{r+1} (sizes round r's filter),
