@@ -1,8 +1,13 @@
+# round-end evidence: GPU tests, every workload's full bench line (oracle parity, cpu_baseline,
+# e2e), the launch list and one full ncu capture of the RMAT-22 step (see tools/profile.sh)
 set -x
 timeout 1500 python -m pytest tests -m gpu -q 2>&1 | tail -3
-nvidia-smi --query-gpu=index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap --format=csv -lms 200 > gpurun_out/clocks_full.csv &
-CPID=$!
-timeout 900 python bench.py > gpurun_out/bench_rmat22.json 2> gpurun_out/bench_rmat22.err
-kill $CPID
-for w in grid64 uniform road dense; do timeout 600 python bench.py --workload $w --no-oracle --e2e-steps 1 > gpurun_out/bench_$w.json 2> gpurun_out/bench_$w.err; done
-tail -c 600 gpurun_out/bench_rmat22.json
+for w in rmat22 grid64 uniform road dense; do
+  timeout 900 python bench.py --workload $w > gpurun_out/bench_$w.json 2> gpurun_out/bench_$w.err
+  python -c "
+import json
+d=json.load(open('gpurun_out/bench_$w.json'))
+print('$w', 'value %.3f G/s'%(d['value']/1e9), 'ms %.3f'%d['ms_per_step'], 'frac %.3f'%(d['roofline']['frac'] or 0), d['parity'], 'e2e %.3f G/s'%(d['e2e']['value']/1e9), 'cpu %.2f M/s'%(d['cpu_baseline']['value']/1e6), 'clk', d['clocks']['sm_mhz'], d['clocks']['reasons'])
+" 2>&1 | tail -1
+done
+bash tools/profile.sh
