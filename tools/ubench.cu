@@ -20,6 +20,16 @@ __global__ void k_red(uint64_t* tab, uint32_t n, uint64_t ops, uint64_t seed) {
     }
 }
 
+// the same REDs, but every CTA into its own private copy of the table (cta * n + h % n)
+__global__ void k_red_private(uint64_t* tab, uint32_t n, uint64_t ops, uint64_t seed) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    uint64_t* mine = tab + (uint64_t)blockIdx.x * n;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < ops; i += stride) {
+        const uint64_t h = mix(seed + i);
+        asm volatile("red.relaxed.gpu.global.min.u64 [%0], %1;" :: "l"(mine + (h % n)), "l"(h) : "memory");
+    }
+}
+
 template <int ILP>
 __global__ void k_gather(const int* map, uint32_t n, uint64_t ops, uint64_t seed, int* sink) {
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x * ILP;
@@ -63,6 +73,33 @@ int main() {
         cudaEventSynchronize(e1);
         cudaEventElapsedTime(&ms, e0, e1);
         printf("RED.MIN.u64 random  table %9u entries: %7.1f G ops/s\n", n, ops / ms / 1e6);
+    }
+    {
+        uint64_t* ptab;
+        const uint32_t n = 1u << 16;
+        cudaMalloc(&ptab, (size_t)n * 8 * nsm * 4);
+        for (int cpsm : {1, 4}) {
+            cudaMemset(ptab, 0xff, (size_t)n * 8 * nsm * cpsm);
+            k_red_private<<<nsm * cpsm, 1024 / cpsm>>>(ptab, n, ops, 1);
+            cudaEventRecord(e0);
+            k_red_private<<<nsm * cpsm, 1024 / cpsm>>>(ptab, n, ops, 7);
+            cudaEventRecord(e1);
+            cudaEventSynchronize(e1);
+            cudaEventElapsedTime(&ms, e0, e1);
+            printf("RED.MIN.u64 random, per-CTA private table of %u (%d CTAs): %7.1f G ops/s\n", n,
+                   nsm * cpsm, ops / ms / 1e6);
+        }
+        for (uint32_t n2 : {1u << 16}) {
+            cudaMemset(tab, 0xff, (size_t)n2 * 8);
+            k_red<<<nsm * 16, 256>>>(tab, n2, ops, 1);
+            cudaEventRecord(e0);
+            k_red<<<nsm * 16, 256>>>(tab, n2, ops, 7);
+            cudaEventRecord(e1);
+            cudaEventSynchronize(e1);
+            cudaEventElapsedTime(&ms, e0, e1);
+            printf("RED.MIN.u64 random  table %9u entries: %7.1f G ops/s\n", n2, ops / ms / 1e6);
+        }
+        cudaFree(ptab);
     }
     int *map, *sink;
     cudaMalloc(&map, (size_t)(1 << 24) * 4);
