@@ -361,7 +361,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     if (g->sim) CKS(galloc(g, &g->shard_best, n * (u64)g->shards.size()));
     CKS(galloc(g, &g->P, n));
     CKS(galloc(g, &g->Mtmp, n));
-    CKS(galloc(g, &g->tcnt, 2 * hook_tiles(n) + 2));
+    CKS(galloc(g, &g->tcnt, 2 * std::max(hook_tiles(n), out_tiles(g->nwords)) + 2));
     CKS(galloc(g, &g->maps, 2 * n + 1));  // sum_r n_r <= 2n: every live component merges
     CKS(galloc(g, &g->msf, g->nwords));
     CKS(galloc(g, &g->phi, n));
@@ -724,8 +724,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     {
         Prof p(g, s, MST_K_OUTPUT, r);
         if (g->nwords) {
-            CK(launch_output(s, (u32)g->nwords, g->msf, out_ids, g->status, g->epoch++,
-                             g->dcnt + C_OUT));
+            CK(launch_output(s, (u32)g->nwords, g->msf, out_ids, g->tcnt, g->dcnt + C_OUT));
         } else {
             CK(cudaMemsetAsync(g->dcnt + C_OUT, 0, sizeof(u32), s));
         }
