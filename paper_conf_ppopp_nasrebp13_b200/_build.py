@@ -51,6 +51,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
            "-Xptxas", "-v" if verbose else "-O3",
            "-I", os.path.join(ROOT, "include"), "-I", inc,
+           *os.environ.get("MST_NVCC_FLAGS", "").split(),  # A/B variants (tools/ab.sh)
            *sources(), "-o", tmp,
            "-L", libdir, "-l:libnccl.so.2", "-Xlinker", f"-rpath={libdir}"]
     r = subprocess.run(cmd, capture_output=True, text=True)
