@@ -150,6 +150,14 @@ def byte_model(st):
     return out
 
 
+def min0_byte_model(st):
+    """Round-0 minimum (A2): 16 B read per edge record; with the light-edge phase also 16 B
+    written per light record (a_r[0] = the records the pass wrote, incl. the dead filler that
+    ends each warp's reserved block)."""
+    light = st.get("light_t", 0xFFFFFFFF) != 0xFFFFFFFF
+    return 16 * st["arcs0"] + (16 * st["a_r"][0] if light and st["rounds"] else 0)
+
+
 def run_gpu(args):
     import torch
     import torch.distributed as dist
@@ -219,6 +227,7 @@ def run_gpu(args):
     #     on the run's stream: per-kernel durations for the roofline and the per-round table
     h.set_profiling(True)
     filt_ms, filt_bytes, filt_launches, prof_ms = 0.0, 0, 0, []
+    min0_ms, min0_bytes, min0_launches = 0.0, 0, 0
     round_acc = None
     for _ in range(args.steps):
         (ids, cnt, tot), ms = timed_step()
@@ -228,6 +237,9 @@ def run_gpu(args):
         filt_launches += st["kernel_launches"]["filter"]
         bm = byte_model(st)
         filt_bytes += sum(x["bytes"] for x in bm if x["kind"] == "filter")
+        min0_ms += st["kernel_ms"]["min0"]
+        min0_launches += st["kernel_launches"]["min0"]
+        min0_bytes += min0_byte_model(st)
         if round_acc is None:
             round_acc = [{"r": r, "kind": bm[r]["kind"], "n_r": st["n_r"][r], "A_r": st["a_r"][r],
                           "compacted": bm[r].get("compacted"),
@@ -278,10 +290,19 @@ def run_gpu(args):
                              f"({cpu_model()}); timer covers key build + sort + union-find + id sort",
                    "seconds": o_secs}
         achieved = filt_bytes / (filt_ms * 1e-3) / 1e9 if filt_ms > 0 else None
+        step_prof = float(np.sum(prof_ms)) if prof_ms else None
+
+        def kernel_roof(name, ms, byts, launches):
+            a = byts / (ms * 1e-3) / 1e9 if ms > 0 else None
+            return {"bound": "hbm", "kernel": name, "achieved": a, "peak": peak, "unit": "GB/s",
+                    "frac": a / peak if a else None, "peak_source": peak_src,
+                    "avg_launch_ms": ms / max(launches, 1), "bytes_per_launch": byts / max(launches, 1),
+                    "share_of_step": ms / step_prof if step_prof else None}
         traffic = None
         tp = os.path.join(ROOT, "profiles", f"ncu_traffic_{args.workload}.json")
         if os.path.exists(tp):
-            traffic = json.load(open(tp)).get("filter_dram_bytes_per_launch")
+            traffic = json.load(open(tp)).get(
+                "filter_dram_bytes_per_launch" if filt_ms >= min0_ms else "min0_dram_bytes_per_launch")
         rounds = []
         for rr in round_acc or []:
             gbs = rr["filter_bytes"] / (rr["filter_ms"] * 1e-3) / 1e9 if rr["filter_ms"] > 0 else None
@@ -300,16 +321,22 @@ def run_gpu(args):
                        "build_ms": build_ms, "gen_s": gen_s},
             "parity": parity,
             "num_edges": cnt, "total_weight": tot,
-            "roofline": {"bound": "hbm", "kernel": "k_arc_pass<MODE_FILTER> (A8)",
-                         "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak if achieved else None, "traffic": traffic,
-                         "peak_source": peak_src,
-                         "avg_launch_ms": filt_ms / max(filt_launches, 1),
-                         "bytes_per_launch": filt_bytes / max(filt_launches, 1),
-                         "share_of_step": filt_ms / float(np.sum(prof_ms)) if prof_ms else None,
+            # the dominant kernel of the step (largest share): the per-round pass (A8) or the
+            # round-0 minimum (A2, which also writes the light records when that phase is on)
+            "roofline": {**(kernel_roof("k_arc_pass<MODE_FILTER> (A8)", filt_ms, filt_bytes,
+                                        filt_launches)
+                            if filt_ms >= min0_ms else
+                            kernel_roof("k_arc_pass<MODE_MIN0> (A2)", min0_ms, min0_bytes,
+                                        min0_launches)),
+                         "traffic": traffic,
                          "timing": "CUDA events around every launch on the run's stream, "
                                    "over a second timed region of the same K steps (value "
                                    "is timed without them)"},
+            "roofline_kernels": {
+                "A8 filter": kernel_roof("k_arc_pass<MODE_FILTER> (A8)", filt_ms, filt_bytes, filt_launches),
+                "A2 min0": kernel_roof("k_arc_pass<MODE_MIN0> (A2)", min0_ms, min0_bytes, min0_launches)},
+            "light_phase": {"t": st["light_t"] if st["light_t"] != 0xFFFFFFFF else None,
+                            "switch_round": st["light_switch_round"]},
             "rounds": rounds,
             "kernel_ms_per_step": {k: v for k, v in st["kernel_ms"].items()},
             "profiled_ms_per_step": float(np.mean(prof_ms)) if prof_ms else None,

@@ -144,6 +144,11 @@ typedef struct {
                                                   compaction decision used (-1: none)      */
     int32_t hub_row;                      /* 1: the dense transition kept the top hub's
                                              matrix row in shared memory (heavy tail)     */
+    int32_t light_switch_round;           /* light-edge phase (MST_OPT_LIGHT_FIRST): round
+                                             whose pass re-read every edge record (the
+                                             heavy ones), -1 = not reached / phase off    */
+    uint32_t light_t;                     /* its weight threshold (light: w <= light_t);
+                                             0xffffffff when the phase was off            */
 } mst_stats;
 
 mst_status mst_get_stats(const mst_graph* g, mst_stats* out);
@@ -172,8 +177,21 @@ mst_status mst_set_profiling(mst_graph* g, int enable);
  *       (deletion deferred to the dense transition). Decided on the device per pass from the
  *       previous pass's exact survival (round 0: 4096 sampled records); never changes the
  *       result.
+ *   MST_OPT_LIGHT_FIRST (default -1 = auto; 0 = off, else K in [1, 64]): light-edge phase
+ *       (auto: K = 4 when there are >= 64 records per vertex, else K = 2). Kruskal
+ *       takes the edges in (w, id) order (the "ordered" algorithm), so the
+ *       forest restricted to the edges with w <= t is the forest of that light subgraph for
+ *       every t. mst_run first picks t so that about K*n edge records are light (a 4096-record
+ *       sample, on the device), writes the light records while it computes the round-0
+ *       minima, runs the Boruvka rounds over the light records only — a component without a
+ *       light edge is deferred, not finished — and once no light edge joins two components
+ *       re-reads every record (relabelled; all the light ones are now intra-component and
+ *       deleted) and continues as usual. Used when at least 2*K*n records exist (dense and
+ *       heavy-tailed inputs), on single-GPU handles without MST_OPT_KEEP_EDGES. Never
+ *       changes the result.
  */
-enum { MST_OPT_DENSE = 1, MST_OPT_KEEP_EDGES = 2, MST_OPT_DEVICE_TAIL = 3, MST_OPT_COMPACT_TAU = 4 };
+enum { MST_OPT_DENSE = 1, MST_OPT_KEEP_EDGES = 2, MST_OPT_DEVICE_TAIL = 3, MST_OPT_COMPACT_TAU = 4,
+       MST_OPT_LIGHT_FIRST = 5 };
 mst_status mst_set_option(mst_graph* g, int option, int64_t value);
 
 /* ------------------------------------------------------------------ multi-GPU (§8(e))

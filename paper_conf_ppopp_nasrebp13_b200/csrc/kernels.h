@@ -49,11 +49,24 @@ cudaError_t launch_owner_degree(cudaStream_t st, int nsm, u32 m, const u32* eu, 
 cudaError_t launch_scatter(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
                            const unsigned* w, u32* cursor, uint4* arcs, uint2* euv,
                            int hi_owner);
+// light_out != nullptr (MST_OPT_LIGHT_FIRST): also append the records of weight <= *light_t
+// to light_out; every consumer warp reserves blocks of light_blk records (one atomic each)
+// and fills the unused end of its last block with dead records (owner ~0); *light_count =
+// records written including that filler (<= light + light_blk * warps of the launch)
 cudaError_t launch_min0(cudaStream_t st, int nsm, u64 A, const uint4* arcs, u64* best, u32 nb,
-                        u32* tile_ctrs, u32 seq);
+                        u32* tile_ctrs, u32 seq, uint4* light_out = nullptr,
+                        const u32* light_t = nullptr, u32* light_count = nullptr,
+                        u32 light_blk = 0);
+u32 pass_warps(int nsm);  // consumer warps of one pass launch (the filler bound)
+// weight threshold t of the light-edge phase: about `target` of the A records have w <= t
+// (binary search on a 4096-record sample); writes *t
+cudaError_t launch_light_threshold(cudaStream_t st, const uint4* arcs, u64 A, u64 target, u32* t);
+// phi[x] = chain.m[len-1][...chain.m[0][x]] for x < n (-1 stays -1)
+cudaError_t launch_chain_compose(cudaStream_t st, int nsm, u32 n, const MapChain& chain, int* phi);
+// defer (light-edge phase): a component with no (light) edge left is kept, not finished
 cudaError_t launch_hook(cudaStream_t st, u32 nr, const u64* best, u64* best_next, u64* hmap, u32 tag,
                         const uint2* euv, const MapChain& chain, u32* P, int* Mtmp, u32* msf,
-                        u64* acc, u32* tcnt, u32* n_next);
+                        u64* acc, u32* tcnt, u32* n_next, bool defer = false);
 // tcnt: 2 * hook_tiles(n) words (tile counts, then their exclusive scan)
 cudaError_t launch_jump(cudaStream_t st, int nsm, u32 nr, u32* P, const int* Mtmp, const u32* tcnt,
                         int* Mr, const u32* nn, u64* best_next, const int* hub, int* hub_next);

@@ -83,7 +83,9 @@ constexpr int C_SEEN = C_TAIL + 1 + MST_MAX_ROUNDS;  // records entering pass r 
 constexpr int C_SURV = C_SEEN + MST_MAX_ROUNDS;       // survivors of pass r (all shards)
 constexpr int C_SAMP = C_SURV + MST_MAX_ROUNDS;       // round-0 sample: {alive, samples}
 constexpr int C_HUB = C_SAMP + 2;  // label of internal vertex 0 (the top hub) per round
-constexpr int DCNT_WORDS = C_HUB + MST_MAX_ROUNDS + 1;
+constexpr int C_LT = C_HUB + MST_MAX_ROUNDS + 1;  // light-edge threshold t
+constexpr u32 LBLK_MIN = 32, LBLK_MAX = 256;      // light write: records per warp reservation
+constexpr int DCNT_WORDS = C_LT + 1;
 constexpr int HSURV = MST_MAX_ROUNDS + 1;  // mapped words: [0, HSURV) sizes, [HSURV, 2 HSURV) decisions
 
 struct Shard {
@@ -137,6 +139,7 @@ struct mst_graph {
     bool opt_keep = false;   // MST_OPT_KEEP_EDGES (paper-faithful ablation)
     bool opt_tail = true;    // MST_OPT_DEVICE_TAIL
     u32 tau = 950;           // MST_OPT_COMPACT_TAU (permille)
+    int light_k = -1;        // MST_OPT_LIGHT_FIRST (-1 auto, 0 off, else light records ~ K n)
     bool hub_row = false;
     u64* trace = nullptr;    // MST_TAIL_TRACE=1 (tools): phase timestamps of the dense tail    // heavy-tailed input: hub row of the dense transition in smem
     int* phi = nullptr;      // composed label map of the records' label space (row A7)
@@ -355,14 +358,19 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
         cap = std::max(cap, hi[j]);
     }
     // ping-pong arc buffers: a shard's arcs keep their [lo, hi) window in every buffer
-    for (int b = 0; b < 2; ++b) CKS(galloc(g, &g->abuf[b], cap));
+    // abuf[0] also takes the light-edge write of a single-GPU handle: the light records plus
+    // at most LBLK_MAX dead filler records per consumer warp (MST_OPT_LIGHT_FIRST)
+    for (int b = 0; b < 2; ++b)
+        CKS(galloc(g, &g->abuf[b], cap + (b == 0 && G == 1 ? (u64)pass_warps(g->nsm) * LBLK_MAX : 0)));
     CKS(galloc(g, &g->bestA, n));
     CKS(galloc(g, &g->bestB, n));
     if (g->sim) CKS(galloc(g, &g->shard_best, n * (u64)g->shards.size()));
     CKS(galloc(g, &g->P, n));
     CKS(galloc(g, &g->Mtmp, n));
     CKS(galloc(g, &g->tcnt, 2 * std::max(hook_tiles(n), out_tiles(g->nwords)) + 2));
-    CKS(galloc(g, &g->maps, 2 * n + 1));  // sum_r n_r <= 2n: every live component merges
+    // sum_r n_r <= 2n when every live component merges each round; the light-edge phase
+    // defers components (no merge) and switches to all edges before 3n + 1 is reached
+    CKS(galloc(g, &g->maps, 3 * n + 1));
     CKS(galloc(g, &g->msf, g->nwords));
     CKS(galloc(g, &g->phi, n));
     if (n >= 2) {  // dense min-matrices (A9 / NEXT-1), <= 67 MB each
@@ -499,15 +507,39 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         CK(cudaMemsetAsync(g->dcnt + C_SEEN, 0, 2 * MST_MAX_ROUNDS * sizeof(u32), s));
         CK(cudaMemsetAsync(g->dcnt + C_HUB, 0, sizeof(u32), s));  // round 0: vertex 0 itself
     }
-    // ---- A2 round-0 minimum (+ A3)
+    // light-edge phase (MST_OPT_LIGHT_FIRST): single handle, enough records to pay
+    static const u32 lk_env = getenv("MST_LIGHT_K") ? (u32)atoi(getenv("MST_LIGHT_K")) : 0xffffffffu;
+    // auto: the light subgraph of a dense near-regular graph must be connected to finish
+    // in the light phase (light degree ~ 2K >= ln n); a heavy-tailed sparse one never is
+    // (low-degree vertices), where fewer light records cost less (measured: dense K = 4,
+    // RMAT-22 K = 2)
+    const u32 lk = lk_env != 0xffffffffu ? lk_env
+                 : g->light_k >= 0 ? (u32)g->light_k : (g->A0 >= 64ull * (u64)n ? 4u : 2u);
+    int phase = (lk > 0 && G == 1 && !g->comm && !g->opt_keep && g->A0 >= 4096 &&
+                 g->A0 >= 2ull * lk * n) ? 1 : 0;
+    g->st.light_switch_round = -1;
+    g->st.light_t = 0xffffffffu;
+    if (phase) {
+        Prof p(g, s, MST_K_MIN0, 0);
+        CK(launch_light_threshold(s, g->arcs0, g->A0, (u64)lk * n, g->dcnt + C_LT));
+    }
+    // ---- A2 round-0 minimum (+ A3); with the light phase it also writes the light records
     for (int j = 0; j < G; ++j) {
         Shard& sh = g->shards[j];
         sh.A = (u32)(sh.hi - sh.lo);
         u64* tgt = g->sim ? g->shard_best + (u64)j * n : g->bestA;
         if (sh.A == 0) continue;
         Prof p(g, s, MST_K_MIN0, 0);
-        CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, (u32)n, g->dcnt + C_TILE,
-                       g->pass_seq++));
+        if (phase) {
+            // a quarter of a warp's expected light records per reservation: few atomics on
+            // the counter, filler <= a quarter of them
+            const u64 per_warp = (u64)lk * n / ((u64)g->nsm * 30);
+            const u32 blk = (u32)std::min<u64>(LBLK_MAX, std::max<u64>(LBLK_MIN, per_warp / 4));
+            CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, (u32)n, g->dcnt + C_TILE,
+                           g->pass_seq++, g->abuf[0], g->dcnt + C_LT, g->dcnt + arec(j, 0), blk));
+        } else
+            CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, (u32)n, g->dcnt + C_TILE,
+                           g->pass_seq++));
     }
     if (g->sim) {
         Prof p(g, s, MST_K_COMM, 0);
@@ -518,8 +550,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     }
 
     // round-0 arc counts (host-known) into the per-round record
-    for (int j = 0; j < G; ++j) g->hcnt[arec(j, 0)] = g->shards[j].A;
-    for (int j = 0; j < G; ++j)
+    for (int j = 0; j < G && !phase; ++j) g->hcnt[arec(j, 0)] = g->shards[j].A;
+    for (int j = 0; j < G && !phase; ++j)
         CK(cudaMemcpyAsync(g->dcnt + arec(j, 0), g->hcnt + arec(j, 0), sizeof(u32),
                            cudaMemcpyHostToDevice, s));
     const u32 tag_base = ((++g->run_seq) & 0xffffffu) << 8;  // run-unique tags for hmap
@@ -533,7 +565,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     // where the alive records live: buffer `cur` (per-shard windows), labels of round `brnd`
     // (n_b = nb_sz labels); a pass whose compaction was decided on the device (sampled) is
     // resolved at the next round's wait (pend)
-    const uint4* cur = g->arcs0;
+    const uint4* cur = phase ? g->abuf[0] : g->arcs0;  // light phase: the light records
     int brnd = 0;
     u32 nb_sz = (u32)n;
     int pend = -1;
@@ -588,7 +620,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         {
             Prof p(g, s, MST_K_HOOK, r);
             CK(launch_hook(s, nr, bcur, bnxt, g->dmap + r, tag_base | (u32)r, g->euv, chain, g->P,
-                           g->Mtmp, g->msf, g->acc, g->tcnt, g->dcnt + C_NNEXT));
+                           g->Mtmp, g->msf, g->acc, g->tcnt, g->dcnt + C_NNEXT,
+                           phase == 1 && r > 0));  // round 0's minima cover every edge
         }
         {   // the jump does not need the host: it reads n_{r+1} on the device and runs
             // while the counts travel to the host
@@ -611,7 +644,26 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             ++r;
             break;
         }
-        if (moff + nr + nn > 2 * n + 1) return fail(MST_EINTERNAL, "label-map storage overflow");
+        if (phase == 1 && (nn == nr || (u64)(nr - nn) * 8 < nr || moff + nr + 3ull * nn > 3 * n)) {
+            // no light edge joins two components any more (every component would otherwise
+            // have merged or absorbed one), or too few merged (most components are deferred:
+            // no light edge), or the label-map storage asks for it: this round's pass
+            // re-reads every edge record in vertex ids through the composed map. Switching
+            // at any round is exact: every merge so far took a component's minimum edge.
+            phase = 2;
+            g->st.light_switch_round = r;
+            if (r >= 2) {
+                Prof p(g, s, MST_K_JUMP, r);
+                CK(launch_chain_compose(s, g->nsm, (u32)n, chain, g->phi));
+            }
+            cur = g->arcs0;
+            brnd = 0;
+            nb_sz = (u32)n;
+            g->hcnt[arec(0, r)] = g->shards[0].A;
+            CK(cudaMemcpyAsync(g->dcnt + arec(0, r), g->hcnt + arec(0, r), sizeof(u32),
+                               cudaMemcpyHostToDevice, s));
+        }
+        if (moff + nr + nn > 3 * n + 1) return fail(MST_EINTERNAL, "label-map storage overflow");
         bool to_dense = false;
         if (dense) {
             // A9/NEXT-1 dense round: scan the matrix, collapse into the next (smaller) one
@@ -619,7 +671,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             CK(launch_dense_init(s, g->nsm, nn, g->mat[mc ^ 1]));
             CK(launch_dense_round(s, g->nsm, nr, g->mat[mc], Mr, nn, g->mat[mc ^ 1], bnxt));
         } else {
-            to_dense = g->mat[0] && g->opt_dense && !g->opt_keep && nn <= (u32)DENSE_MAX;
+            to_dense = g->mat[0] && g->opt_dense && !g->opt_keep && nn <= (u32)DENSE_MAX &&
+                       phase != 1;
             if (to_dense) CK(launch_dense_init(s, g->nsm, nn, g->mat[0]));
             // A7: the map of this round's pass, from the records' label space (round brnd)
             // to round r+1: M_r itself, or composed over the rounds that did not compact
@@ -731,7 +784,9 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     }
     CK(cudaMemcpyAsync(g->hcnt, g->dcnt, 2 * sizeof(u32), cudaMemcpyDeviceToHost, s));
     CK(cudaMemcpyAsync(g->hacc, g->acc, 2 * ACC_SLOTS * sizeof(u64), cudaMemcpyDeviceToHost, s));
+    if (phase) CK(cudaMemcpyAsync(g->hcnt + C_LT, g->dcnt + C_LT, sizeof(u32), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
+    if (phase) g->st.light_t = g->hcnt[C_LT];
     if (pend >= 0) {  // the last sampled decision (stats only)
         u32 word;
         CKS(wait_word(g, s, HSURV + pend, tag_base | (u32)pend, &word));
@@ -947,6 +1002,12 @@ mst_status mst_set_option(mst_graph* g, int option, int64_t value) {
             if (value < 0 || value > 1000)
                 return fail(MST_EINVAL, "MST_OPT_COMPACT_TAU must be in [0, 1000] (permille)");
             g->tau = (u32)value;
+            return MST_OK;
+        }
+        if (option == MST_OPT_LIGHT_FIRST) {
+            if (value < -1 || value > 64)
+                return fail(MST_EINVAL, "MST_OPT_LIGHT_FIRST must be -1 (auto) or in [0, 64]");
+            g->light_k = (int)value;
             return MST_OK;
         }
         if (value != 0 && value != 1) return fail(MST_EINVAL, "option value must be 0 or 1");

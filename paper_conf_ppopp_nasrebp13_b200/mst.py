@@ -28,6 +28,7 @@ EXPORTS = ["mst_create", "mst_create_host", "mst_run", "mst_run_host", "mst_solv
            "mst_get_unique_id", "mst_create_dist", "mst_create_sim", "mst_version",
            "mst_set_option"]
 MST_OPT_DENSE, MST_OPT_KEEP_EDGES, MST_OPT_DEVICE_TAIL, MST_OPT_COMPACT_TAU = 1, 2, 3, 4
+MST_OPT_LIGHT_FIRST = 5
 
 
 class mst_stats(ctypes.Structure):
@@ -45,6 +46,8 @@ class mst_stats(ctypes.Structure):
         ("compacted_mask", ctypes.c_int64),
         ("survival_permille", ctypes.c_int32 * MAX_ROUNDS),
         ("hub_row", ctypes.c_int32),
+        ("light_switch_round", ctypes.c_int32),
+        ("light_t", ctypes.c_uint32),
     ]
 
 
@@ -184,7 +187,8 @@ class MSTGraph:
         return out[: cnt.value], int(cnt.value), int(tot.value)
 
     def set_option(self, option: int, value: int):
-        """mst_set_option: MST_OPT_DENSE / _KEEP_EDGES / _DEVICE_TAIL / _COMPACT_TAU (include/mst.h)."""
+        """mst_set_option: MST_OPT_DENSE / _KEEP_EDGES / _DEVICE_TAIL / _COMPACT_TAU / _LIGHT_FIRST
+        (include/mst.h)."""
         _check(load().mst_set_option(self._h, int(option), int(value)))
 
     def set_profiling(self, on: bool):
@@ -208,6 +212,8 @@ class MSTGraph:
             "compacted": [bool((s.compacted_mask >> r) & 1) for r in range(R)],
             "survival_permille": list(s.survival_permille[:R]),
             "hub_row": bool(s.hub_row),
+            "light_switch_round": s.light_switch_round,
+            "light_t": s.light_t,
         }
 
     def debug_filter_pass(self, map_kind=0, group=1, iters=5, stream=None):

@@ -10,6 +10,7 @@ import mstcheck as mc
 
 torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
+LF = 5  # MST_OPT_LIGHT_FIRST (include/mst.h)
 
 
 @pytest.fixture(scope="module")
@@ -266,7 +267,7 @@ def test_compaction_policy(lib, oracle_mod, gg, k, sd, tau):
     g = gg.config(k, s=7, scale_down=sd)
     for extra in ([], [(lib.mst.MST_OPT_DENSE, 0)]):
         st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, runs=2,
-                           options=[(lib.mst.MST_OPT_COMPACT_TAU, tau)] + extra)
+                           options=[(lib.mst.MST_OPT_COMPACT_TAU, tau), (LF, 0)] + extra)
         sparse = [r for r in range(st["rounds"] - 1)
                   if st["dense_round"] < 0 or r + 1 < st["dense_round"]]
         if tau == 0:
@@ -319,7 +320,7 @@ def test_dense_rounds_used(lib, oracle_mod, gg, k, sd, tail):
     """dense rounds both in the cooperative device tail and as per-round launches"""
     g = gg.config(k, s=3, scale_down=sd)
     st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, runs=2,
-                       options=[(lib.mst.MST_OPT_DEVICE_TAIL, tail)])
+                       options=[(lib.mst.MST_OPT_DEVICE_TAIL, tail), (LF, 0)])
     assert st["dense_round"] >= 0
     assert st["n_r"][-1] <= 1 or st["rounds"] >= 1
 
@@ -344,3 +345,71 @@ def test_dist_single_rank_nccl(lib, oracle_mod, gg, k, sd):
             assert np.array_equal(ids.cpu().numpy(), o_ids) and tot == o_tot
         st = h.stats()
         assert st["nranks"] == 1 and st["kernel_launches"]["comm"] >= 1
+
+
+# ------------------------------------------------------------------ light-edge phase
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_light_first_random_dense(lib, oracle_mod, seed):
+    """dense random multigraphs (m/n 10..60) with the light-edge phase at several K: ties at
+    the threshold (few distinct weights), loops, parallels, several components"""
+    rng = np.random.default_rng(7000 + seed)
+    n = int(rng.integers(300, 6000))
+    m = int(n * rng.integers(10, 60))
+    wmax = [0, 1, 7, 1000, 2**32 - 1, 3][seed % 6]
+    src, dst, w = mc.random_multigraph(rng, n, m, wmax)
+    if seed % 4 == 3:  # a second part joined to nothing: two big components
+        src = np.concatenate([src, src + n]); dst = np.concatenate([dst, dst + n])
+        w = np.concatenate([w, w]); n *= 2
+    K = [1, 2, 4][seed % 3]
+    st = assert_parity(lib, oracle_mod, n, src, dst, w, runs=2, options=[(LF, K)])
+    assert st["light_t"] != 0xFFFFFFFF
+
+
+def test_light_first_deferred_components(lib, oracle_mod):
+    """a light core plus pendant vertices and a whole second core reachable only through
+    heavy edges: components without a light edge are deferred through the light phase and
+    merged after the heavy records are re-read"""
+    rng = np.random.default_rng(5)
+    n1, n2, np_ = 4000, 3000, 2000
+    n = n1 + n2 + np_
+    m1 = 40 * n1
+    s1 = rng.integers(0, n1, m1); d1 = rng.integers(0, n1, m1); w1 = rng.integers(0, 100, m1)
+    m2 = 40 * n2
+    s2 = n1 + rng.integers(0, n2, m2); d2 = n1 + rng.integers(0, n2, m2)
+    w2 = rng.integers(900, 1000, m2)                              # second core: heavy only
+    sp = np.arange(n1 + n2, n); dp = rng.integers(0, n1 + n2, np_)
+    wp = rng.integers(800, 1000, np_)                              # pendants: heavy only
+    sb = rng.integers(0, n1, 50); db = n1 + rng.integers(0, n2, 50)
+    wb = rng.integers(950, 1000, 50)                               # bridges: heavy
+    src = np.concatenate([s1, s2, sp, sb]).astype(np.int32)
+    dst = np.concatenate([d1, d2, dp, db]).astype(np.int32)
+    w = np.concatenate([w1, w2, wp, wb]).astype(np.uint32)
+    for K in (1, 4):
+        st = assert_parity(lib, oracle_mod, n, src, dst, w, runs=2, options=[(LF, K)])
+        assert st["light_t"] < 900 and st["light_switch_round"] >= 1
+
+
+@pytest.mark.parametrize("K", [0, 1, 4, 16])
+@pytest.mark.parametrize("k,sd", [(4, 6), (5, 6), (5, 4), (4, 4)])
+def test_light_first_configs(lib, oracle_mod, gg, k, sd, K):
+    g = gg.config(k, s=2, scale_down=sd)
+    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, runs=2, options=[(LF, K)])
+    assert (st["light_t"] == 0xFFFFFFFF) == (K == 0 or st["arcs0"] < 2 * K * g.n)
+
+
+@pytest.mark.parametrize("opts", [[(1, 0)], [(3, 0)], [(4, 0)], [(4, 1000)], [(1, 0), (4, 0)]])
+def test_light_first_with_other_options(lib, oracle_mod, gg, opts):
+    g = gg.config(5, s=3, scale_down=5)
+    assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, runs=2, options=[(LF, 2)] + opts)
+
+
+def test_light_first_option_range(lib, gg):
+    g = gg.config(1)
+    with lib.MSTGraph(g.n, dev(g.src), dev(g.dst), dev(g.w)) as h:
+        for bad in (-2, 65):
+            with pytest.raises(lib.MSTError):
+                h.set_option(LF, bad)
+        h.set_option(LF, 64)
+        h.set_option(LF, -1)
