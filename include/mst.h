@@ -186,7 +186,7 @@ mst_status mst_set_profiling(mst_graph* g, int enable);
  *       minima, runs the Boruvka rounds over the light records only — a component without a
  *       light edge is deferred, not finished — and once no light edge joins two components
  *       re-reads every record (relabelled; all the light ones are now intra-component and
- *       deleted) and continues as usual. Used when at least 2*K*n records exist (dense and
+ *       deleted) and continues as usual. Used when at least 4*K*n records exist (dense and
  *       heavy-tailed inputs), on single-GPU handles without MST_OPT_KEEP_EDGES. Never
  *       changes the result.
  */

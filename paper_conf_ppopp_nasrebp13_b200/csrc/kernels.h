@@ -57,6 +57,10 @@ cudaError_t launch_min0(cudaStream_t st, int nsm, u64 A, const uint4* arcs, u64*
                         u32* tile_ctrs, u32 seq, uint4* light_out = nullptr,
                         const u32* light_t = nullptr, u32* light_count = nullptr,
                         u32 light_blk = 0);
+// light_blk | 1 << 31: extract only (no minima; light-only round 0)
+// round-0 minimum over records whose count is on the device (*a_in <= a_max)
+cudaError_t launch_min0_dev(cudaStream_t st, int nsm, const u32* a_in, u64 a_max,
+                            const uint4* arcs, u64* best, u32 nb, u32* tile_ctrs, u32 seq);
 u32 pass_warps(int nsm);  // consumer warps of one pass launch (the filler bound)
 // weight threshold t of the light-edge phase: about `target` of the A records have w <= t
 // (binary search on a 4096-record sample); writes *t

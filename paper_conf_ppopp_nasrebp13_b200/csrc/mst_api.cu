@@ -513,10 +513,18 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     // in the light phase (light degree ~ 2K >= ln n); a heavy-tailed sparse one never is
     // (low-degree vertices), where fewer light records cost less (measured: dense K = 4,
     // RMAT-22 K = 2)
+    // light-only round 0 (auto, >= 64 records per vertex): the round-0 pass only extracts
+    // the light records (no minima over the full stream); the round-0 minima come from the
+    // light records and vertices without one are deferred. K = 8 makes that a ~e^-16 event
+    // per vertex on near-regular graphs (light degree ~ Poisson(2K)); it stays exact anyway.
+    static const char* lo_env = getenv("MST_LIGHT_ONLY0");
+    const bool dense_regime = g->A0 >= 64ull * (u64)n;
+    const bool lo0_want = lo_env ? lo_env[0] == '1' : (g->light_k < 0 && dense_regime);
     const u32 lk = lk_env != 0xffffffffu ? lk_env
-                 : g->light_k >= 0 ? (u32)g->light_k : (g->A0 >= 64ull * (u64)n ? 4u : 2u);
+                 : g->light_k >= 0 ? (u32)g->light_k : (lo0_want ? 8u : 2u);
     int phase = (lk > 0 && G == 1 && !g->comm && !g->opt_keep && g->A0 >= 4096 &&
-                 g->A0 >= 2ull * lk * n) ? 1 : 0;
+                 g->A0 >= 4ull * lk * n) ? 1 : 0;  // light records <= a quarter
+    const bool light_only0 = lo0_want && phase;
     g->st.light_switch_round = -1;
     g->st.light_t = 0xffffffffu;
     if (phase) {
@@ -536,7 +544,12 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             const u64 per_warp = (u64)lk * n / ((u64)g->nsm * 30);
             const u32 blk = (u32)std::min<u64>(LBLK_MAX, std::max<u64>(LBLK_MIN, per_warp / 4));
             CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, (u32)n, g->dcnt + C_TILE,
-                           g->pass_seq++, g->abuf[0], g->dcnt + C_LT, g->dcnt + arec(j, 0), blk));
+                           g->pass_seq++, g->abuf[0], g->dcnt + C_LT, g->dcnt + arec(j, 0),
+                           blk | (light_only0 ? 1u << 31 : 0u)));
+            if (light_only0)
+                CK(launch_min0_dev(s, g->nsm, g->dcnt + arec(j, 0),
+                                   sh.A + (u64)pass_warps(g->nsm) * LBLK_MAX, g->abuf[0], tgt,
+                                   (u32)n, g->dcnt + C_TILE, g->pass_seq++));
         } else
             CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, (u32)n, g->dcnt + C_TILE,
                            g->pass_seq++));
@@ -621,7 +634,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             Prof p(g, s, MST_K_HOOK, r);
             CK(launch_hook(s, nr, bcur, bnxt, g->dmap + r, tag_base | (u32)r, g->euv, chain, g->P,
                            g->Mtmp, g->msf, g->acc, g->tcnt, g->dcnt + C_NNEXT,
-                           phase == 1 && r > 0));  // round 0's minima cover every edge
+                           phase == 1 && (r > 0 || light_only0)));  // (else round 0's
+                                                                 // minima cover every edge)
         }
         {   // the jump does not need the host: it reads n_{r+1} on the device and runs
             // while the counts travel to the host
@@ -646,7 +660,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         }
         if (phase == 1 && (nn == nr || (u64)(nr - nn) * 8 < nr || moff + nr + 3ull * nn > 3 * n)) {
             // no light edge joins two components any more (every component would otherwise
-            // have merged or absorbed one), or too few merged (most components are deferred:
+            // have merged or absorbed one), or < 1/8 merged (most components are deferred:
             // no light edge), or the label-map storage asks for it: this round's pass
             // re-reads every edge record in vertex ids through the composed map. Switching
             // at any round is exact: every merge so far took a component's minimum edge.
@@ -685,7 +699,10 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             }
             // compaction policy: never (keep-edges: the paper's scheme, or tau = 0), always
             // (tau >= 1000), or decided on the device from the estimated survival (CompactCtl)
-            const bool never = g->opt_keep || g->tau == 0;
+            // the pass that re-reads every record after the light phase never compacts:
+            // measured on RMAT-22, ~70 % of the records still join two components there, but
+            // one more hook round usually finishes (writing them back cost 0.3 ms)
+            const bool never = g->opt_keep || g->tau == 0 || r == g->st.light_switch_round;
             int dsh = -1;  // the shard whose pass reports the device-side decision
             for (int j = 0; j < G && dsh < 0; ++j)
                 if (g->shards[j].hi > g->shards[j].lo) dsh = j;

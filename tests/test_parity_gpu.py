@@ -355,14 +355,14 @@ def test_light_first_random_dense(lib, oracle_mod, seed):
     """dense random multigraphs (m/n 10..60) with the light-edge phase at several K: ties at
     the threshold (few distinct weights), loops, parallels, several components"""
     rng = np.random.default_rng(7000 + seed)
+    K = [1, 2, 4][seed % 3]
     n = int(rng.integers(300, 6000))
-    m = int(n * rng.integers(10, 60))
+    m = int(n * rng.integers(4 * K + 1, 60))
     wmax = [0, 1, 7, 1000, 2**32 - 1, 3][seed % 6]
     src, dst, w = mc.random_multigraph(rng, n, m, wmax)
     if seed % 4 == 3:  # a second part joined to nothing: two big components
         src = np.concatenate([src, src + n]); dst = np.concatenate([dst, dst + n])
         w = np.concatenate([w, w]); n *= 2
-    K = [1, 2, 4][seed % 3]
     st = assert_parity(lib, oracle_mod, n, src, dst, w, runs=2, options=[(LF, K)])
     assert st["light_t"] != 0xFFFFFFFF
 
@@ -396,7 +396,7 @@ def test_light_first_deferred_components(lib, oracle_mod):
 def test_light_first_configs(lib, oracle_mod, gg, k, sd, K):
     g = gg.config(k, s=2, scale_down=sd)
     st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, runs=2, options=[(LF, K)])
-    assert (st["light_t"] == 0xFFFFFFFF) == (K == 0 or st["arcs0"] < 2 * K * g.n)
+    assert (st["light_t"] == 0xFFFFFFFF) == (K == 0 or st["arcs0"] < 4 * K * g.n)
 
 
 @pytest.mark.parametrize("opts", [[(1, 0)], [(3, 0)], [(4, 0)], [(4, 1000)], [(1, 0), (4, 0)]])
@@ -413,3 +413,21 @@ def test_light_first_option_range(lib, gg):
                 h.set_option(LF, bad)
         h.set_option(LF, 64)
         h.set_option(LF, -1)
+
+
+def test_light_only_round0_deferred(lib, oracle_mod):
+    """dense regime (>= 64 records per vertex, auto options): round 0 reads only the light
+    records; pendant vertices whose edges are all heavy are deferred from round 0 on and get
+    their edge after the switch to all records; isolated vertices finish"""
+    rng = np.random.default_rng(11)
+    nc, npend, niso = 3000, 500, 50
+    n = nc + npend + niso
+    mc_ = 100 * nc
+    s1 = rng.integers(0, nc, mc_); d1 = rng.integers(0, nc, mc_); w1 = rng.integers(0, 100, mc_)
+    sp = np.repeat(np.arange(nc, nc + npend), 2); dp = rng.integers(0, nc, 2 * npend)
+    wp = rng.integers(900, 1000, 2 * npend)
+    src = np.concatenate([s1, sp]).astype(np.int32)
+    dst = np.concatenate([d1, dp]).astype(np.int32)
+    w = np.concatenate([w1, wp]).astype(np.uint32)
+    st = assert_parity(lib, oracle_mod, n, src, dst, w, runs=2)
+    assert st["light_t"] < 900 and st["light_switch_round"] >= 0

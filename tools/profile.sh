@@ -1,10 +1,26 @@
-# launch list (cold-cache, serialised; compare SHARES) + one full capture of the RMAT-22 step
+# launch list (cold-cache, serialised; compare SHARES) + one full capture of one mst_run step
 WL=${WL:-rmat22}
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_$WL.csv \
     python bench.py --workload $WL --steps 2 --warmup 3 --e2e-steps 0 --no-oracle > /dev/null 2>&1
-# warmup 3 + 1 timed step: skip the warmup runs' launches of the captured kernels
-ncu --set full --clock-control none --import-source on \
-    -k regex:"arc_pass|k_hook|k_jump|k_dense|k_output|k_sample|k_compose" -s 45 -c 15 \
-    -o gpurun_out/full_$WL python bench.py --workload $WL --steps 1 --warmup 3 --e2e-steps 0 --no-oracle \
+# the bench runs warmup + 2 x steps mst_run calls: capture the kernels of the LAST run only
+RE='arc_pass|k_hook|k_jump|k_dense|k_output|k_out_|k_sample|k_compose|k_light|k_chain'
+SKIP=$(python - "$WL" "$RE" <<'PY'
+import csv, re, sys
+wl, rx = sys.argv[1], re.compile(sys.argv[2])
+rows = [r for r in csv.reader(open(f"gpurun_out/launches_{wl}.csv")) if len(r) > 5]
+h = rows[0]; k = h.index("Kernel Name"); idc = h.index("ID")
+seen = {}
+for r in rows[1:]:
+    seen.setdefault(r[idc], r[k])
+hits = [n for n in seen.values() if rx.search(n)]
+runs = 3 + 2 * 2  # warmup + 2 timed + 2 profiled steps (profile.sh --steps 2 --warmup 3)
+per = len(hits) // runs
+print((runs - 1) * per, per)
+PY
+)
+set -- $SKIP
+ncu --set full --clock-control none --import-source on -k regex:"$RE" -s $1 -c $2 \
+    -o gpurun_out/full_$WL python bench.py --workload $WL --steps 2 --warmup 3 --e2e-steps 0 --no-oracle \
     > gpurun_out/ncu_full_$WL.log 2>&1
 tail -1 gpurun_out/ncu_full_$WL.log
+python tools/ncu_traffic.py gpurun_out/full_$WL.ncu-rep $WL "tools/profile.sh WL=$WL" > /dev/null
