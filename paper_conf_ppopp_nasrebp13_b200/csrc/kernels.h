@@ -48,7 +48,7 @@ cudaError_t launch_owner_degree(cudaStream_t st, int nsm, u32 m, const u32* eu, 
                                 u32* odeg, int hi_owner);
 cudaError_t launch_scatter(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
                            const unsigned* w, u32* cursor, uint4* arcs, uint2* euv,
-                           int hi_owner);
+                           int hi_owner, u32* wmax);
 // light_out != nullptr (MST_OPT_LIGHT_FIRST): also append the records of weight <= *light_t
 // to light_out; every consumer warp reserves blocks of light_blk records (one atomic each)
 // and fills the unused end of its last block with dead records (owner ~0); *light_count =
@@ -56,11 +56,12 @@ cudaError_t launch_scatter(cudaStream_t st, int nsm, u32 m, const u32* eu, const
 cudaError_t launch_min0(cudaStream_t st, int nsm, u64 A, const uint4* arcs, u64* best, u32 nb,
                         u32* tile_ctrs, u32 seq, uint4* light_out = nullptr,
                         const u32* light_t = nullptr, u32* light_count = nullptr,
-                        u32 light_blk = 0);
+                        u32 light_blk = 0, u32 kfmt = 0);
 // light_blk | 1 << 31: extract only (no minima; light-only round 0)
 // round-0 minimum over records whose count is on the device (*a_in <= a_max)
 cudaError_t launch_min0_dev(cudaStream_t st, int nsm, const u32* a_in, u64 a_max,
-                            const uint4* arcs, u64* best, u32 nb, u32* tile_ctrs, u32 seq);
+                            const uint4* arcs, u64* best, u32 nb, u32* tile_ctrs, u32 seq,
+                            u32 kfmt = 0);
 u32 pass_warps(int nsm);  // consumer warps of one pass launch (the filler bound)
 // weight threshold t of the light-edge phase: about `target` of the A records have w <= t
 // (binary search on a 4096-record sample); writes *t
@@ -70,7 +71,7 @@ cudaError_t launch_chain_compose(cudaStream_t st, int nsm, u32 n, const MapChain
 // defer (light-edge phase): a component with no (light) edge left is kept, not finished
 cudaError_t launch_hook(cudaStream_t st, u32 nr, const u64* best, u64* best_next, u64* hmap, u32 tag,
                         const uint2* euv, const MapChain& chain, u32* P, int* Mtmp, u32* msf,
-                        u64* acc, u32* tcnt, u32* n_next, bool defer = false);
+                        u64* acc, u32* tcnt, u32* n_next, bool defer = false, u32 kfmt = 0);
 // tcnt: 2 * hook_tiles(n) words (tile counts, then their exclusive scan)
 cudaError_t launch_jump(cudaStream_t st, int nsm, u32 nr, u32* P, const int* Mtmp, const u32* tcnt,
                         int* Mr, const u32* nn, u64* best_next, const int* hub, int* hub_next);
@@ -79,7 +80,8 @@ cudaError_t launch_filter_min(cudaStream_t st, int nsm, const u32* a_in, u64 a_m
                               const uint4* in, const int* M, uint4* out, u64* best, u32 nb,
                               u64* status, u32 epoch, u32* a_next, u32* tile_ctrs, u32 seq,
                               u64* mat, const CompactCtl& cc = CompactCtl(),
-                              const int* hub = nullptr);
+                              const int* hub = nullptr, u32 kfmt = 0);
+// kfmt: key format of the minima the pass emits = s1 | pb << 8 (pb = 0: (w << 32) | eid)
 cudaError_t launch_dense_best(cudaStream_t st, int nsm, u32 n, const u64* mat, u64* best);
 cudaError_t launch_dense_init(cudaStream_t st, int nsm, u32 n, u64* mat);
 cudaError_t launch_dense_round(cudaStream_t st, int nsm, u32 n, const u64* mat, const int* M,

@@ -84,8 +84,9 @@ constexpr int C_SURV = C_SEEN + MST_MAX_ROUNDS;       // survivors of pass r (al
 constexpr int C_SAMP = C_SURV + MST_MAX_ROUNDS;       // round-0 sample: {alive, samples}
 constexpr int C_HUB = C_SAMP + 2;  // label of internal vertex 0 (the top hub) per round
 constexpr int C_LT = C_HUB + MST_MAX_ROUNDS + 1;  // light-edge threshold t
+constexpr int C_WMAX = C_LT + 1;                   // largest weight (build)
 constexpr u32 LBLK_MIN = 32, LBLK_MAX = 256;      // light write: records per warp reservation
-constexpr int DCNT_WORDS = C_LT + 1;
+constexpr int DCNT_WORDS = C_WMAX + 1;
 constexpr int HSURV = MST_MAX_ROUNDS + 1;  // mapped words: [0, HSURV) sizes, [HSURV, 2 HSURV) decisions
 
 struct Shard {
@@ -140,6 +141,7 @@ struct mst_graph {
     bool opt_tail = true;    // MST_OPT_DEVICE_TAIL
     u32 tau = 950;           // MST_OPT_COMPACT_TAU (permille)
     int light_k = -1;        // MST_OPT_LIGHT_FIRST (-1 auto, 0 off, else light records ~ K n)
+    u32 kfmt = 0;            // packed minima keys (w << s1 | eid << pb | partner): s1 | pb << 8
     bool hub_row = false;
     u64* trace = nullptr;    // MST_TAIL_TRACE=1 (tools): phase timestamps of the dense tail    // heavy-tailed input: hub row of the dense transition in smem
     int* phi = nullptr;      // composed label map of the records' label space (row A7)
@@ -344,7 +346,8 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     g->A0 = A0;
     CKS(galloc(g, &g->arcs0, A0));
     CKS(galloc(g, &g->euv, m));
-    CK(launch_scatter(g->cst, g->nsm, (u32)m, g->eu, g->ev, w, cursor, g->arcs0, g->euv, hi_owner));
+    CK(launch_scatter(g->cst, g->nsm, (u32)m, g->eu, g->ev, w, cursor, g->arcs0, g->euv, hi_owner,
+                      g->dcnt + C_WMAX));
 
     // shards: simulation = all G ranges locally; distributed = this rank's range only
     const int G = nshards_sim > 1 ? nshards_sim : nranks;
@@ -377,7 +380,17 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
         CKS(galloc(g, &g->mat[0], dense_entries(n)));
         CKS(galloc(g, &g->mat[1], dense_entries(n)));
     }
+    CK(cudaMemcpyAsync(g->hcnt + C_WMAX, g->dcnt + C_WMAX, sizeof(u32), cudaMemcpyDeviceToHost,
+                       g->cst));
     CK(cudaStreamSynchronize(g->cst));
+    {   // packed minima keys when weight, edge id and a label fit in 63 bits (not with dist,
+        // whose per-round allreduce is format-agnostic anyway; kept simple)
+        auto bits = [](u64 x) { u32 b = 0; while (x) { ++b; x >>= 1; } return b; };
+        const u32 wb = bits(g->hcnt[C_WMAX]), eb = bits(m > 0 ? (u64)m - 1 : 0),
+                  pb = bits(n > 0 ? (u64)n - 1 : 0);
+        static const char* pk = getenv("MST_PACKED_KEYS");  // "0": always (w << 32) | eid
+        if (pb > 0 && wb + eb + pb <= 63 && !(pk && pk[0] == '0')) g->kfmt = (eb + pb) | (pb << 8);
+    }
     g->st.n = g->n;
     g->st.m = g->m;
     g->st.arcs0 = (int64_t)g->A0;
@@ -545,14 +558,14 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             const u32 blk = (u32)std::min<u64>(LBLK_MAX, std::max<u64>(LBLK_MIN, per_warp / 4));
             CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, (u32)n, g->dcnt + C_TILE,
                            g->pass_seq++, g->abuf[0], g->dcnt + C_LT, g->dcnt + arec(j, 0),
-                           blk | (light_only0 ? 1u << 31 : 0u)));
+                           blk | (light_only0 ? 1u << 31 : 0u), g->kfmt));
             if (light_only0)
                 CK(launch_min0_dev(s, g->nsm, g->dcnt + arec(j, 0),
                                    sh.A + (u64)pass_warps(g->nsm) * LBLK_MAX, g->abuf[0], tgt,
-                                   (u32)n, g->dcnt + C_TILE, g->pass_seq++));
+                                   (u32)n, g->dcnt + C_TILE, g->pass_seq++, g->kfmt));
         } else
             CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, (u32)n, g->dcnt + C_TILE,
-                           g->pass_seq++));
+                           g->pass_seq++, nullptr, nullptr, nullptr, 0, g->kfmt));
     }
     if (g->sim) {
         Prof p(g, s, MST_K_COMM, 0);
@@ -634,8 +647,9 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             Prof p(g, s, MST_K_HOOK, r);
             CK(launch_hook(s, nr, bcur, bnxt, g->dmap + r, tag_base | (u32)r, g->euv, chain, g->P,
                            g->Mtmp, g->msf, g->acc, g->tcnt, g->dcnt + C_NNEXT,
-                           phase == 1 && (r > 0 || light_only0)));  // (else round 0's
-                                                                 // minima cover every edge)
+                           phase == 1 && (r > 0 || light_only0),  // (else round 0's
+                                                                  // minima cover every edge)
+                           dense ? 0u : g->kfmt));  // dense rounds: matrix keys (w << 32 | eid)
         }
         {   // the jump does not need the host: it reads n_{r+1} on the device and runs
             // while the counts travel to the host
@@ -740,7 +754,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                                      g->dcnt + arec(j, r + 1), g->dcnt + C_TILE, g->pass_seq++,
                                      to_dense ? g->mat[0] : nullptr, ccj,
                                      (to_dense && use_hub_row(g))
-                                         ? (const int*)g->dcnt + C_HUB + r + 1 : nullptr));
+                                         ? (const int*)g->dcnt + C_HUB + r + 1 : nullptr,
+                                     g->kfmt));
             }
             if (to_dense && use_hub_row(g)) g->st.hub_row = 1;
             if (adaptive) {
