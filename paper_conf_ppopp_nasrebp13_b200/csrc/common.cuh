@@ -82,6 +82,13 @@ __device__ __forceinline__ u32 ld_relaxed_u32(const u32* p) {
     asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
+// Plain (weak, L1-cacheable) load of a word other threads may update in this kernel: only
+// for monotone data where a stale value is still correct (pointer-jumping ancestors).
+__device__ __forceinline__ u32 ld_weak_u32(const u32* p) {
+    u32 v;
+    asm volatile("ld.global.u32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
 __device__ __forceinline__ void st_relaxed_u32(u32* p, u32 v) {
     asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
 }
