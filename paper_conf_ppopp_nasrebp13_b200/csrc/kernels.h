@@ -89,7 +89,8 @@ cudaError_t launch_dense_round(cudaStream_t st, int nsm, u32 n, const u64* mat, 
 u64 dense_entries(u64 n);
 cudaError_t launch_dense_tail(cudaStream_t st, int nsm, u32 n0, u64* best0, u64* best1,
                               u64* mat0, u64* mat1, const uint2* euv, const MapChain& chain,
-                              u32* msf, u64* acc, u32* bar, u32* stats, u64* trace = nullptr);
+                              u32* msf, u64* acc, u32* bar, u32* stats, u64* trace = nullptr,
+                              int defer = 0, int* map_out = nullptr, u32* n_out = nullptr);
 cudaError_t launch_compose(cudaStream_t st, int nsm, u32 nb, const int* src, const int* Mr, int* phi);
 cudaError_t launch_sample_survival(cudaStream_t st, const uint4* in, const u32* a_ptr, const int* M,
                                    u32* num, u32* den);

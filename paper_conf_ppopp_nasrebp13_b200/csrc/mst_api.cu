@@ -85,8 +85,9 @@ constexpr int C_SAMP = C_SURV + MST_MAX_ROUNDS;       // round-0 sample: {alive,
 constexpr int C_HUB = C_SAMP + 2;  // label of internal vertex 0 (the top hub) per round
 constexpr int C_LT = C_HUB + MST_MAX_ROUNDS + 1;  // light-edge threshold t
 constexpr int C_WMAX = C_LT + 1;                   // largest weight (build)
+constexpr int C_TAILN = C_WMAX + 1;                // light-phase tail: labels after it
 constexpr u32 LBLK_MIN = 32, LBLK_MAX = 256;      // light write: records per warp reservation
-constexpr int DCNT_WORDS = C_WMAX + 1;
+constexpr int DCNT_WORDS = C_TAILN + 1;
 constexpr int HSURV = MST_MAX_ROUNDS + 1;  // mapped words: [0, HSURV) sizes, [HSURV, 2 HSURV) decisions
 
 struct Shard {
@@ -613,6 +614,10 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     int mc = 0;
     g->st.dense_round = -1;
     int tail_r0 = -1;  // first round run by the device-resident dense tail
+    // a light-phase tail that stopped on deferred components hands over a virtual round: its
+    // composite map (tail-start labels -> labels after it) and size, with no hook to run
+    bool vround = false, hub_ok = true;
+    u32 v_nn = 0;
     while (true) {
         if (r >= MST_MAX_ROUNDS || chain.len >= MST_CHAIN_MAX)
             return fail(MST_EINTERNAL, "round limit exceeded (r = %d)", r);
@@ -624,9 +629,12 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                 CK(cudaMalloc(&g->trace, 64 * sizeof(u64)));
                 CK(cudaMemsetAsync(g->trace, 0, 64 * sizeof(u64), s));
             }
+            const bool lp = phase == 1;
+            if (lp && moff + nr > 3 * n + 1) return fail(MST_EINTERNAL, "label-map storage overflow");
             CK(launch_dense_tail(s, g->nsm, nr, bcur, bnxt, g->mat[mc], g->mat[mc ^ 1], g->euv,
                                  chain, g->msf, g->acc, g->dcnt + C_BAR, g->dcnt + C_TAIL,
-                                 tr ? g->trace : nullptr));
+                                 tr ? g->trace : nullptr, lp ? 1 : 0,
+                                 lp ? g->maps + moff : nullptr, lp ? g->dcnt + C_TAILN : nullptr));
             if (tr) {
                 u64 h[64];
                 CK(cudaMemcpyAsync(h, g->trace, sizeof h, cudaMemcpyDeviceToHost, s));
@@ -639,10 +647,38 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                 }
                 CK(cudaMemsetAsync(g->trace, 0, 64 * sizeof(u64), s));
             }
-            tail_r0 = r;
-            break;
+            if (lp) {  // did the light phase finish inside the tail?
+                CK(cudaMemcpyAsync(g->hcnt + C_TAIL, g->dcnt + C_TAIL,
+                                   (1 + MST_MAX_ROUNDS) * sizeof(u32), cudaMemcpyDeviceToHost, s));
+                CK(cudaMemcpyAsync(g->hcnt + C_TAILN, g->dcnt + C_TAILN, sizeof(u32),
+                                   cudaMemcpyDeviceToHost, s));
+                CK(cudaStreamSynchronize(s));
+                const u32 k = g->hcnt[C_TAIL];
+                const u32 nf = g->hcnt[C_TAILN];
+                if (k >= 1 && nf > 1 && r + (int)k < MST_MAX_ROUNDS) {
+                    for (u32 i = 0; i < k; ++i) {
+                        g->st.n_r[r + i] = g->hcnt[C_TAIL + 1 + i];
+                        g->st.a_r[r + i] = (int64_t)dense_entries(g->hcnt[C_TAIL + 1 + i]);
+                    }
+                    r += (int)k - 1;  // this iteration stands for the tail's last round
+                    vround = true;
+                    v_nn = nf;
+                    hub_ok = false;  // (the hub's label is not tracked through the tail)
+                    CK(cudaMemsetAsync(bnxt, 0xff, (size_t)nf * sizeof(u64), s));
+                }
+            }
+            if (!vround) {
+                tail_r0 = r;
+                break;
+            }
         }
         int* Mr = g->maps + moff;
+        u32 nn;
+        const bool was_v = vround;
+        if (vround) {
+            vround = false;
+            nn = v_nn;
+        } else {
         {
             Prof p(g, s, MST_K_HOOK, r);
             CK(launch_hook(s, nr, bcur, bnxt, g->dmap + r, tag_base | (u32)r, g->euv, chain, g->P,
@@ -659,7 +695,6 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         }
         // one host round trip per round: n_{r+1} (sizes round r's filter),
         // read zero-copy from the word the hook's last tile writes to mapped host memory
-        u32 nn;
         CKS(wait_round(g, s, r, tag_base | (u32)r, &nn));
         g->st.n_r[r] = nr;
         g->st.a_r[r] = dense ? (int64_t)dense_entries(nr) : -1;  // sparse: filled at the end
@@ -668,17 +703,20 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             CKS(wait_word(g, s, HSURV + pend, tag_base | (u32)pend, &word));
             resolve(word);
         }
+        }
         if (nn <= 1) {  // <= 1 live component left: no inter-component edge remains
             ++r;
             break;
         }
-        if (phase == 1 && (nn == nr || (u64)(nr - nn) * 8 < nr || moff + nr + 3ull * nn > 3 * n)) {
+        if (phase == 1 && (was_v || nn == nr || (u64)(nr - nn) * 8 < nr ||
+                           moff + nr + 3ull * nn > 3 * n)) {
             // no light edge joins two components any more (every component would otherwise
             // have merged or absorbed one), or < 1/8 merged (most components are deferred:
             // no light edge), or the label-map storage asks for it: this round's pass
             // re-reads every edge record in vertex ids through the composed map. Switching
             // at any round is exact: every merge so far took a component's minimum edge.
             phase = 2;
+            dense = false;  // the records are read again (a dense phase-1 matrix is dropped)
             g->st.light_switch_round = r;
             if (r >= 2) {
                 Prof p(g, s, MST_K_JUMP, r);
@@ -699,8 +737,10 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             CK(launch_dense_init(s, g->nsm, nn, g->mat[mc ^ 1]));
             CK(launch_dense_round(s, g->nsm, nr, g->mat[mc], Mr, nn, g->mat[mc ^ 1], bnxt));
         } else {
+            // (light phase: only when its ~K n records outnumber the matrix cells — measured
+            // on dense: 0.76 M light records against 5.7 M cells made the tail 2x slower)
             to_dense = g->mat[0] && g->opt_dense && !g->opt_keep && nn <= (u32)DENSE_MAX &&
-                       phase != 1;
+                       (phase != 1 || (u64)lk * n >= dense_entries(nn));
             if (to_dense) CK(launch_dense_init(s, g->nsm, nn, g->mat[0]));
             // A7: the map of this round's pass, from the records' label space (round brnd)
             // to round r+1: M_r itself, or composed over the rounds that did not compact
@@ -753,11 +793,11 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                                      Mpass, out, tgt, nn, g->status, g->epoch++,
                                      g->dcnt + arec(j, r + 1), g->dcnt + C_TILE, g->pass_seq++,
                                      to_dense ? g->mat[0] : nullptr, ccj,
-                                     (to_dense && use_hub_row(g))
+                                     (to_dense && use_hub_row(g) && hub_ok)
                                          ? (const int*)g->dcnt + C_HUB + r + 1 : nullptr,
                                      g->kfmt));
             }
-            if (to_dense && use_hub_row(g)) g->st.hub_row = 1;
+            if (to_dense && use_hub_row(g) && hub_ok) g->st.hub_row = 1;
             if (adaptive) {
                 pend = r;
                 pend_out = outbuf;
