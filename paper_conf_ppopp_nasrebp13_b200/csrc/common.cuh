@@ -199,6 +199,7 @@ __device__ __forceinline__ void mbar_arrive(u64* bar) {
 }
 __device__ __forceinline__ void mbar_wait(u64* bar, u32 parity) {
     const u32 a = smem_addr(bar);
+
     asm volatile(
         "{\n"
         ".reg .pred P1;\n"
