@@ -73,8 +73,11 @@ cudaError_t launch_hook(cudaStream_t st, u32 nr, const u64* best, u64* best_next
                         const uint2* euv, const MapChain& chain, u32* P, int* Mtmp, u32* msf,
                         u64* acc, u32* tcnt, u32* n_next, bool defer = false, u32 kfmt = 0);
 // tcnt: 2 * hook_tiles(n) words (tile counts, then their exclusive scan)
+// rounds with few hook tiles: the jump also does k_hook_scan's work (n_{r+1} to *nn and to
+// the tagged word hmap, which launch_hook then does not launch)
 cudaError_t launch_jump(cudaStream_t st, int nsm, u32 nr, u32* P, const int* Mtmp, const u32* tcnt,
-                        int* Mr, const u32* nn, u64* best_next, const int* hub, int* hub_next);
+                        int* Mr, u32* nn, u64* best_next, const int* hub, int* hub_next,
+                        u64* hmap, u32 tag);
 u64 hook_tiles(u64 n);
 cudaError_t launch_filter_min(cudaStream_t st, int nsm, const u32* a_in, u64 a_max,
                               const uint4* in, const int* M, uint4* out, u64* best, u32 nb,

@@ -691,7 +691,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             // while the counts travel to the host
             Prof p(g, s, MST_K_JUMP, r);
             CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, g->tcnt, Mr, g->dcnt + C_NNEXT, bnxt,
-                           (const int*)g->dcnt + C_HUB + r, (int*)g->dcnt + C_HUB + r + 1));
+                           (const int*)g->dcnt + C_HUB + r, (int*)g->dcnt + C_HUB + r + 1,
+                           g->dmap + r, tag_base | (u32)r));
         }
         // one host round trip per round: n_{r+1} (sizes round r's filter),
         // read zero-copy from the word the hook's last tile writes to mapped host memory
