@@ -616,7 +616,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     int tail_r0 = -1;  // first round run by the device-resident dense tail
     // a light-phase tail that stopped on deferred components hands over a virtual round: its
     // composite map (tail-start labels -> labels after it) and size, with no hook to run
-    bool vround = false, hub_ok = true;
+    bool vround = false, hub_ok = true, phi_ready = false;
     u32 v_nn = 0;
     while (true) {
         if (r >= MST_MAX_ROUNDS || chain.len >= MST_CHAIN_MAX)
@@ -719,9 +719,12 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             phase = 2;
             dense = false;  // the records are read again (a dense phase-1 matrix is dropped)
             g->st.light_switch_round = r;
-            if (r >= 2) {
+            if (r >= 1 && chain.len + 1 < MST_CHAIN_MAX) {  // Ψ = Mr ∘ chain in one kernel
                 Prof p(g, s, MST_K_JUMP, r);
-                CK(launch_chain_compose(s, g->nsm, (u32)n, chain, g->phi));
+                MapChain full = chain;
+                full.m[full.len++] = Mr;
+                CK(launch_chain_compose(s, g->nsm, (u32)n, full, g->phi));
+                phi_ready = true;
             }
             cur = g->arcs0;
             brnd = 0;
@@ -746,7 +749,10 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             // A7: the map of this round's pass, from the records' label space (round brnd)
             // to round r+1: M_r itself, or composed over the rounds that did not compact
             const int* Mpass = Mr;
-            if (brnd < r) {
+            if (phi_ready) {  // (the switch composed the whole chain with M_r already)
+                Mpass = g->phi;
+                phi_ready = false;
+            } else if (brnd < r) {
                 Prof p(g, s, MST_K_JUMP, r);
                 const int* src = (brnd == r - 1) ? chain.m[chain.len - 1] : g->phi;
                 CK(launch_compose(s, g->nsm, nb_sz, src, Mr, g->phi));
