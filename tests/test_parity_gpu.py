@@ -431,3 +431,30 @@ def test_light_only_round0_deferred(lib, oracle_mod):
     w = np.concatenate([w1, wp]).astype(np.uint32)
     st = assert_parity(lib, oracle_mod, n, src, dst, w, runs=2)
     assert st["light_t"] < 900 and st["light_switch_round"] >= 0
+
+
+@pytest.mark.parametrize("nclusters", [60, 140, 400, 900])
+def test_transition_into_few_components(lib, oracle_mod, nclusters):
+    """many records between few components at the dense transition: the whole next matrix in
+    shared memory (<= ~157 components), local rows + warp-merged REDs (<= 1024), with and
+    without the hub row (a hub joined to everything by heavy edges makes degrees heavy-tailed)"""
+    rng = np.random.default_rng(nclusters)
+    size = 40
+    n = nclusters * size + 1
+    base = 1 + np.arange(nclusters) * size
+    # light edges inside clusters (each cluster contracts in the first rounds)
+    ci = rng.integers(0, nclusters, 60 * nclusters)
+    s1 = base[ci] + rng.integers(0, size, ci.size); d1 = base[ci] + rng.integers(0, size, ci.size)
+    w1 = rng.integers(0, 100, ci.size)
+    # many medium edges between clusters (the records that cross at the transition)
+    ca, cb = rng.integers(0, nclusters, 400 * nclusters), rng.integers(0, nclusters, 400 * nclusters)
+    s2 = base[ca] + rng.integers(0, size, ca.size); d2 = base[cb] + rng.integers(0, size, cb.size)
+    w2 = rng.integers(100, 900, ca.size)
+    # the hub: vertex 0 joined to every vertex by heavy edges
+    s3 = np.zeros(n - 1, np.int64); d3 = np.arange(1, n); w3 = rng.integers(900, 1000, n - 1)
+    src = np.concatenate([s1, s2, s3]).astype(np.int32)
+    dst = np.concatenate([d1, d2, d3]).astype(np.int32)
+    w = np.concatenate([w1, w2, w3]).astype(np.uint32)
+    for opts in ([(LF, 0)], [(LF, 0), (lib.mst.MST_OPT_DEVICE_TAIL, 0)], []):
+        st = assert_parity(lib, oracle_mod, n, src, dst, w, runs=2, options=opts)
+    assert st["rounds"] >= 2
