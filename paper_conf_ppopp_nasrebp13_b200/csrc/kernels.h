@@ -62,7 +62,11 @@ cudaError_t launch_min0(cudaStream_t st, int nsm, u64 A, const uint4* arcs, u64*
 cudaError_t launch_min0_dev(cudaStream_t st, int nsm, const u32* a_in, u64 a_max,
                             const uint4* arcs, u64* best, u32 nb, u32* tile_ctrs, u32 seq,
                             u32 kfmt = 0);
-u32 pass_warps(int nsm);  // consumer warps of one pass launch (the filler bound)
+u32 pass_warps(int nsm);
+unsigned long long kernel_launches();  // kernels launched by this process so far
+// A1: best = inf (n), msf = 0 (nwords), acc = 0 (nacc), ctr = 0 (nctr), *zero1 = *zero2 = 0
+cudaError_t launch_init(cudaStream_t st, int nsm, u32 n, u64* best, u32 nwords, u32* msf,
+                        u64* acc, u32 nacc, u32* ctr, u32 nctr, u32* zero1, u32* zero2);  // consumer warps of one pass launch (the filler bound)
 // weight threshold t of the light-edge phase: about `target` of the A records have w <= t
 // (binary search on a 4096-record sample); writes *t
 cudaError_t launch_light_threshold(cudaStream_t st, const uint4* arcs, u64 A, u64 target, u32* t);

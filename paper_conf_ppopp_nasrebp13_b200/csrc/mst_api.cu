@@ -219,7 +219,6 @@ struct Prof {
             a = next_event(g);
             cudaEventRecord(a, s);
         }
-        g->st.gpu_launches++;
     }
     ~Prof() {
         if (g->prof) {
@@ -494,6 +493,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     g->recs.clear();
     g->evused = 0;
     g->st.gpu_launches = 0;
+    const unsigned long long kl0 = kernel_launches();  // kernels of this run (set at the end)
     g->st.rounds = 0;
     for (int j = 0; j < MST_K_COUNT; ++j) {
         g->st.kernel_ms[j] = 0;
@@ -514,12 +514,13 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     // ---- A1 init
     {
         Prof p(g, s, MST_K_INIT, 0);
-        CK(cudaMemsetAsync(g->bestA, 0xff, n * sizeof(u64), s));
-        CK(cudaMemsetAsync(g->msf, 0, std::max<u64>(g->nwords, 1) * sizeof(u32), s));
-        CK(cudaMemsetAsync(g->acc, 0, 2 * ACC_SLOTS * sizeof(u64), s));
+        // best_0 = inf, forest bits, accumulators, per-pass counters (C_SEEN, C_SURV), the
+        // hub label (round 0: vertex 0 itself) and shard 0's round-0 record count
+        static_assert(C_SURV == C_SEEN + MST_MAX_ROUNDS, "counter layout");
+        CK(launch_init(s, g->nsm, (u32)n, g->bestA, (u32)std::max<u64>(g->nwords, 1), g->msf,
+                       g->acc, 2 * ACC_SLOTS, g->dcnt + C_SEEN, 2 * MST_MAX_ROUNDS,
+                       g->dcnt + C_HUB, g->dcnt + arec(0, 0)));
         if (g->sim) CK(cudaMemsetAsync(g->shard_best, 0xff, n * G * sizeof(u64), s));
-        CK(cudaMemsetAsync(g->dcnt + C_SEEN, 0, 2 * MST_MAX_ROUNDS * sizeof(u32), s));
-        CK(cudaMemsetAsync(g->dcnt + C_HUB, 0, sizeof(u32), s));  // round 0: vertex 0 itself
     }
     // light-edge phase (MST_OPT_LIGHT_FIRST): single handle, enough records to pay
     static const u32 lk_env = getenv("MST_LIGHT_K") ? (u32)atoi(getenv("MST_LIGHT_K")) : 0xffffffffu;
@@ -909,6 +910,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         }
     }
     g->st.profiling = g->prof ? 1 : 0;
+    g->st.gpu_launches = (int64_t)(kernel_launches() - kl0);
     return MST_OK;
 }
 

@@ -68,6 +68,7 @@ def test_grid64(lib, oracle_mod, gg):
     g = gg.config(1)
     st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, runs=3)
     assert st["rounds"] >= 3
+    assert st["gpu_launches"] >= st["rounds"]  # every kernel of the run is counted
 
 
 @pytest.mark.parametrize("seed", range(120))
