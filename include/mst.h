@@ -175,8 +175,9 @@ mst_status mst_set_profiling(mst_graph* g, int enable);
  *       records that survive is below tau/1000; otherwise the next pass re-reads the same
  *       records through the composed label map (row A7). 1000 = always compact, 0 = never
  *       (deletion deferred to the dense transition). Decided on the device per pass from the
- *       previous pass's exact survival (round 0: 4096 sampled records); never changes the
- *       result.
+ *       previous pass's exact survival (round 0: 4096 sampled records); the passes of the
+ *       light-edge phase and the pass that then re-reads every record never compact. Never
+ *       changes the result.
  *   MST_OPT_LIGHT_FIRST (default -1 = auto; 0 = off, else K in [1, 64]): light-edge phase
  *       (auto: K = 4 when there are >= 64 records per vertex, else K = 2). Kruskal
  *       takes the edges in (w, id) order (the "ordered" algorithm), so the

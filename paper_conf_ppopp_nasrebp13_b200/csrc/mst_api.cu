@@ -764,7 +764,10 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             // the pass that re-reads every record after the light phase never compacts:
             // measured on RMAT-22, ~70 % of the records still join two components there, but
             // one more hook round usually finishes (writing them back cost 0.3 ms)
-            const bool never = g->opt_keep || g->tau == 0 || r == g->st.light_switch_round;
+            // (nor do the light-phase passes: their records are read only a couple more
+            // times; measured on RMAT-22 with ~80 % surviving: 49.2 -> 51.1 G edges/s)
+            const bool never = g->opt_keep || g->tau == 0 || r == g->st.light_switch_round ||
+                               phase == 1;
             int dsh = -1;  // the shard whose pass reports the device-side decision
             for (int j = 0; j < G && dsh < 0; ++j)
                 if (g->shards[j].hi > g->shards[j].lo) dsh = j;
