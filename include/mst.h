@@ -170,7 +170,7 @@ mst_status mst_set_profiling(mst_graph* g, int enable);
  *       morph step (deletion) buys.
  *   MST_OPT_DEVICE_TAIL (default 1): once dense, run every remaining round inside one
  *       cooperative kernel (no host round trip per round); 0 = one launch set per round.
- *   MST_OPT_COMPACT_TAU (default 950, permille in [0, 1000]): a sparse pass deletes the dead
+ *   MST_OPT_COMPACT_TAU (default 900, permille in [0, 1000]): a sparse pass deletes the dead
  *       edge records (compaction, the morph step) only when the sampled fraction of its
  *       records that survive is below tau/1000; otherwise the next pass re-reads the same
  *       records through the composed label map (row A7). 1000 = always compact, 0 = never

@@ -140,7 +140,7 @@ struct mst_graph {
     bool opt_dense = true;   // MST_OPT_DENSE
     bool opt_keep = false;   // MST_OPT_KEEP_EDGES (paper-faithful ablation)
     bool opt_tail = true;    // MST_OPT_DEVICE_TAIL
-    u32 tau = 950;           // MST_OPT_COMPACT_TAU (permille)
+    u32 tau = 900;           // MST_OPT_COMPACT_TAU (permille; measured: uniform 950 -> 900 +2.7 %)
     int light_k = -1;        // MST_OPT_LIGHT_FIRST (-1 auto, 0 off, else light records ~ K n)
     u32 kfmt = 0;            // packed minima keys (w << s1 | eid << pb | partner): s1 | pb << 8
     bool hub_row = false;
