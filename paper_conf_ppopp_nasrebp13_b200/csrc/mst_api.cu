@@ -710,7 +710,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             ++r;
             break;
         }
-        if (phase == 1 && (was_v || nn == nr || (u64)(nr - nn) * 8 < nr ||
+        static const u64 sw_den = getenv("MST_LIGHT_SWITCH") ? (u64)atoi(getenv("MST_LIGHT_SWITCH")) : 8;
+        if (phase == 1 && (was_v || nn == nr || (u64)(nr - nn) * sw_den < nr ||
                            moff + nr + 3ull * nn > 3 * n)) {
             // no light edge joins two components any more (every component would otherwise
             // have merged or absorbed one), or < 1/8 merged (most components are deferred:
