@@ -459,3 +459,24 @@ def test_transition_into_few_components(lib, oracle_mod, nclusters):
     for opts in ([(LF, 0)], [(LF, 0), (lib.mst.MST_OPT_DEVICE_TAIL, 0)], []):
         st = assert_parity(lib, oracle_mod, n, src, dst, w, runs=2, options=opts)
     assert st["rounds"] >= 2
+
+
+@pytest.mark.parametrize("seed", range(16))
+def test_light_auto_dense_regime_random(lib, oracle_mod, seed):
+    """default options on random multigraphs with >= 64 records per vertex: light-only round 0
+    (K = 8) with ties at the threshold, loops, parallels, disconnected parts and vertices whose
+    edges are all heavy"""
+    rng = np.random.default_rng(9100 + seed)
+    n = int(rng.integers(200, 3000))
+    m = int(n * rng.choice([70, 100, 200]))
+    wmax = [0, 2, 9, 1000, 2**32 - 1, 50][seed % 6]
+    src, dst, w = mc.random_multigraph(rng, n, m, wmax)
+    if seed % 3 == 0:  # a few vertices whose edges are all much heavier
+        k = max(1, n // 50)
+        hv = rng.choice(n, k, replace=False)
+        heavy = np.isin(src, hv) | np.isin(dst, hv)
+        w = np.where(heavy, np.uint32(min(2**32 - 1, int(wmax) * 4 + 100)), w).astype(np.uint32)
+    if seed % 4 == 1:  # plus a separate small dense part
+        src = np.concatenate([src, (src[:m // 8] % 64) + n]); dst = np.concatenate([dst, (dst[:m // 8] % 64) + n])
+        w = np.concatenate([w, w[:m // 8]]); n += 64
+    assert_parity(lib, oracle_mod, n, src, dst, w, runs=2)
