@@ -101,8 +101,9 @@ cudaError_t launch_dense_tail(cudaStream_t st, int nsm, u32 n0, u64* best0, u64*
 cudaError_t launch_compose(cudaStream_t st, int nsm, u32 nb, const int* src, const int* Mr, int* phi);
 cudaError_t launch_sample_survival(cudaStream_t st, const uint4* in, const u32* a_ptr, const int* M,
                                    u32* num, u32* den);
+// max_ids: an upper bound of the forest size (n - 1) — sizes the staging of the id writes
 cudaError_t launch_output(cudaStream_t st, u32 nwords, const u32* msf, int* out, u32* tcnt,
-                          u32* out_count);
+                          u32* out_count, u32 max_ids);
 u64 out_tiles(u64 nwords);  // tcnt needs 2 * out_tiles(nwords) words
 cudaError_t launch_combine_min(cudaStream_t st, int nsm, u32 nr, int nshards, u64* shard_best,
                                u64 stride, u64* best);

@@ -861,7 +861,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     {
         Prof p(g, s, MST_K_OUTPUT, r);
         if (g->nwords) {
-            CK(launch_output(s, (u32)g->nwords, g->msf, out_ids, g->tcnt, g->dcnt + C_OUT));
+            CK(launch_output(s, (u32)g->nwords, g->msf, out_ids, g->tcnt, g->dcnt + C_OUT,
+                             (u32)std::max<int64_t>(n - 1, 1)));
         } else {
             CK(cudaMemsetAsync(g->dcnt + C_OUT, 0, sizeof(u32), s));
         }

@@ -480,3 +480,18 @@ def test_light_auto_dense_regime_random(lib, oracle_mod, seed):
         src = np.concatenate([src, (src[:m // 8] % 64) + n]); dst = np.concatenate([dst, (dst[:m // 8] % 64) + n])
         w = np.concatenate([w, w[:m // 8]]); n += 64
     assert_parity(lib, oracle_mod, n, src, dst, w, runs=2)
+
+
+def test_output_dense_forest_tiles(lib, oracle_mod):
+    """forest edges packed into the first edge ids (a path listed first, then many heavier
+    edges): the output's id staging is sized to the average forest density, so these tiles
+    exceed it and take the direct-store path"""
+    rng = np.random.default_rng(17)
+    n = 300_000
+    ps = np.arange(n - 1, dtype=np.int64)
+    extra = 4_000_000
+    es = rng.integers(0, n, extra); ed = rng.integers(0, n, extra)
+    src = np.concatenate([ps, es]).astype(np.int32)
+    dst = np.concatenate([ps + 1, ed]).astype(np.int32)
+    w = np.concatenate([rng.integers(0, 10, n - 1), rng.integers(10, 1000, extra)]).astype(np.uint32)
+    assert_parity(lib, oracle_mod, n, src, dst, w, runs=2)
