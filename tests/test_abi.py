@@ -56,3 +56,30 @@ def test_product_path_does_not_import_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
                 txt = open(os.path.join(dirpath, f)).read()
                 assert not bad.search(txt), f
+
+
+def test_stats_struct_and_options_match_the_header(tmp_path):
+    """the ctypes mirror of mst_stats and the option numbers agree with include/mst.h (a
+    plain C compile of the header measures the struct)"""
+    import subprocess
+    import ctypes as C
+    import paper_conf_ppopp_nasrebp13_b200 as p
+    src = tmp_path / "probe.c"
+    src.write_text('#include <stdio.h>\n#include <stddef.h>\n#include "mst.h"\n'
+                   'int main(void){printf("%zu %zu %zu %d %d %d %d %d\\n", sizeof(mst_stats),'
+                   ' offsetof(mst_stats, light_switch_round), offsetof(mst_stats, light_t),'
+                   ' MST_OPT_DENSE, MST_OPT_KEEP_EDGES, MST_OPT_DEVICE_TAIL, MST_OPT_COMPACT_TAU,'
+                   ' MST_OPT_LIGHT_FIRST); return 0;}\n')
+    exe = tmp_path / "probe"
+    r = subprocess.run(["gcc", "-I", os.path.join(ROOT, "include"), "-I", "/usr/local/cuda/include",
+                        str(src), "-o", str(exe)], capture_output=True, text=True)
+    assert r.returncode == 0, r.stderr
+    vals = subprocess.run([str(exe)], capture_output=True, text=True).stdout.split()
+    size, off_sw, off_t = (int(x) for x in vals[:3])
+    S = p.mst.mst_stats
+    assert C.sizeof(S) == size
+    assert S.light_switch_round.offset == off_sw and S.light_t.offset == off_t
+    m = p.mst
+    assert [int(x) for x in vals[3:]] == [m.MST_OPT_DENSE, m.MST_OPT_KEEP_EDGES,
+                                          m.MST_OPT_DEVICE_TAIL, m.MST_OPT_COMPACT_TAU,
+                                          m.MST_OPT_LIGHT_FIRST]
