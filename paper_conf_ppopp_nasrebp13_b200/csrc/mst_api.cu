@@ -544,7 +544,18 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     g->st.light_t = 0xffffffffu;
     if (phase) {
         Prof p(g, s, MST_K_MIN0, 0);
-        CK(launch_light_threshold(s, g->arcs0, g->A0, (u64)lk * n, g->dcnt + C_LT));
+        static const char* tf = getenv("MST_LIGHT_T");  // ablation: a fixed threshold
+        if (tf) {
+            g->hcnt[C_LT] = (u32)strtoul(tf, nullptr, 10);
+            CK(cudaMemcpyAsync(g->dcnt + C_LT, g->hcnt + C_LT, sizeof(u32), cudaMemcpyHostToDevice, s));
+        } else {
+            // auto K = 2 aims a little above 2 n: below t ~ 119 RMAT-22 leaves a small part
+            // uncontracted after the all-records pass (one more full pass: 52.7 -> 44.4 G
+            // edges/s) while t 120-150 is flat; the 4096-record sample puts t within ~+-5
+            const bool auto_k = lk_env == 0xffffffffu && g->light_k < 0 && !lo0_want;
+            const u64 target = auto_k ? (u64)23 * n / 10 : (u64)lk * n;
+            CK(launch_light_threshold(s, g->arcs0, g->A0, target, g->dcnt + C_LT));
+        }
     }
     // ---- A2 round-0 minimum (+ A3); with the light phase it also writes the light records
     for (int j = 0; j < G; ++j) {
