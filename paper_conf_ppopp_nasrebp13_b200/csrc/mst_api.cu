@@ -552,8 +552,10 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             // auto K = 2 aims a little above 2 n: below t ~ 119 RMAT-22 leaves a small part
             // uncontracted after the all-records pass (one more full pass: 52.7 -> 44.4 G
             // edges/s) while t 120-150 is flat; the 4096-record sample puts t within ~+-5
-            const bool auto_k = lk_env == 0xffffffffu && g->light_k < 0 && !lo0_want;
-            const u64 target = auto_k ? (u64)23 * n / 10 : (u64)lk * n;
+            // (dense regime, K = 8: aimed at 10 n so that t <= 2 — light degree ~8, a few
+            // vertices without a light edge and one more all-records pass — stays unlikely)
+            const bool auto_k = lk_env == 0xffffffffu && g->light_k < 0;
+            const u64 target = !auto_k ? (u64)lk * n : lo0_want ? (u64)10 * n : (u64)23 * n / 10;
             CK(launch_light_threshold(s, g->arcs0, g->A0, target, g->dcnt + C_LT));
         }
     }
