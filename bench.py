@@ -377,10 +377,11 @@ def run_reference(args):
     val = m_s * args.steps / tot
     sample = (f"{'full workload' if m_s == g.m else 'edge-id prefix'} ({m_s} of {g.m} edges) "
               f"per step; 1 of {cpu_cores()} host cores ({cpu_model()})")
-    return {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": 0, "steps": args.steps,
+    return {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": tot * 1e3 / args.steps,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "u64", "data": "synthetic", "impl": "reference",
+            "device": "host cpu (the oracle; rank 0 only, the GPUs are idle)",
             "config": {"workload": g.name, "n": g.n, "m": g.m, "sample_m": m_s},
             "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
                              "sample": sample},
