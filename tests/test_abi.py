@@ -83,3 +83,43 @@ def test_stats_struct_and_options_match_the_header(tmp_path):
     assert [int(x) for x in vals[3:]] == [m.MST_OPT_DENSE, m.MST_OPT_KEEP_EDGES,
                                           m.MST_OPT_DEVICE_TAIL, m.MST_OPT_COMPACT_TAU,
                                           m.MST_OPT_LIGHT_FIRST]
+
+
+def test_argument_errors_before_any_device_work():
+    """include/mst.h error conventions on the host-side checks: MST_EINVAL with a message for
+    out-of-range sizes, null pointers and null handles — decided before any CUDA call, so they
+    hold on a machine without a GPU too; mst_destroy(NULL) is a no-op"""
+    import ctypes as C
+    import paper_conf_ppopp_nasrebp13_b200 as p
+    L = p.load()
+    EINVAL = 1
+    g = C.c_void_p()
+    buf = (C.c_int32 * 4)(0, 1, 1, 2)
+    wb = (C.c_uint32 * 2)(1, 1)
+    cases = [
+        (1 << 31, 2, buf, buf, wb, "n ="),            # n > 2^31 - 1
+        (-1, 2, buf, buf, wb, "n ="),
+        (4, 1 << 31, buf, buf, wb, "m ="),            # m > 2^31 - 1
+        (4, -5, buf, buf, wb, "m ="),
+        (4, 2, None, buf, wb, "null input pointer"),
+        (4, 2, buf, buf, None, "null input pointer"),
+        (0, 2, buf, buf, wb, "n = 0"),                # edges on no vertices
+    ]
+    for create in (L.mst_create, L.mst_create_host):
+        for n, m, s, d, w, msg in cases:
+            st = create(n, m, s, d, w, C.byref(g))
+            assert st == EINVAL, (create, n, m, st)
+            assert msg in L.mst_last_error().decode(), L.mst_last_error()
+            assert not g.value  # *out is NULL after a failed create
+        assert create(4, 2, buf, buf, wb, None) == EINVAL  # out == NULL
+    ne, tw = C.c_int64(), C.c_uint64()
+    assert L.mst_run(None, None, buf, C.byref(ne), C.byref(tw)) == EINVAL
+    assert L.mst_run_host(None, None, buf, C.byref(ne), C.byref(tw)) == EINVAL
+    assert L.mst_set_option(None, p.mst.MST_OPT_DENSE, 1) == EINVAL
+    assert L.mst_set_profiling(None, 1) == EINVAL
+    assert L.mst_get_stats(None, C.byref(p.mst.mst_stats())) == EINVAL
+    L.mst_destroy(None)
+    out_ids = (C.c_int32 * 4)()
+    assert L.mst_solve_host(-1, 0, None, None, None, out_ids, C.byref(ne), C.byref(tw)) == EINVAL
+    assert L.mst_create_sim(4, 2, buf, buf, wb, 0, C.byref(g)) == EINVAL  # nshards < 1
+    assert L.mst_create_sim(4, 2, buf, buf, wb, 65, C.byref(g)) == EINVAL  # nshards > 64
