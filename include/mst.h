@@ -52,16 +52,22 @@ typedef enum {
 typedef struct mst_graph mst_graph; /* opaque; owned by the library */
 
 /* ------------------------------------------------------------------ build (row A0)
- * mst_create — validate the COO input and build the device-resident arc arrays.
+ * mst_create — validate the COO input and build the device-resident edge records.
  *   n, m     : vertex and edge counts (see conventions).
  *   src, dst : DEVICE pointers, int32[m], caller-owned, read only during the call.
  *   w        : DEVICE pointer, uint32[m], caller-owned, read only during the call.
  *   out      : receives the handle; *out = NULL on any error (nothing is leaked).
- * Builds the CSR of PAPER.md §6 L229 ("store each edge twice, once for each direction"):
- * 2 arcs per non-self-loop edge, grouped by source vertex, each carrying the packed key
- * (uint64(w) << 32 | e). All per-round buffers are allocated here once, sized for the
- * worst case (§7.1: MST pre-allocation, "the sum of the nodes in all
- * components is constant"); mst_run allocates nothing. Synchronous. */
+ * The call first synchronises the device (cudaDeviceSynchronize), so inputs still being
+ * written by work in flight on any stream are complete before the build reads them.
+ * Layout (reading R14): the CSR of PAPER.md §6 L229 stores "each edge twice,
+ * once for each direction"; this build stores every non-self-loop edge ONCE, as a 16-byte
+ * record {owner, other, eid, w} in the segment of its owner endpoint (the higher internal
+ * vertex id under the build's hub-first numbering), records grouped by owner (CSR order).
+ * E_0 = the number of non-self-loop edges = the records built (mst_stats.arcs0). Both
+ * endpoints' minima are still computed every round, so the result is the same. All per-round
+ * buffers are allocated here once, sized for the worst case (§7.1: MST
+ * pre-allocation, "the sum of the nodes in all components is constant"); mst_run allocates
+ * nothing. Synchronous. */
 mst_status mst_create(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                       const uint32_t* w, mst_graph** out);
 
@@ -124,12 +130,14 @@ enum {
     MST_K_COUNT = 8
 };
 typedef struct {
-    int64_t n, m, arcs0;                  /* vertices, edges, A_0 = 2 * #non-loop edges  */
+    int64_t n, m, arcs0;                  /* vertices, edges, E_0 = #non-loop edges (one
+                                             record per edge, all ranks together)         */
     int32_t rounds;                       /* R: rounds executed by the last run          */
     int32_t nranks, rank;                 /* 1/0 for single-GPU handles                  */
-    int64_t local_arcs0;                  /* arcs owned by this rank                     */
+    int64_t local_arcs0;                  /* edge records owned by this rank             */
     int64_t n_r[MST_MAX_ROUNDS];          /* live components entering round r            */
-    int64_t a_r[MST_MAX_ROUNDS];          /* alive (local) arcs entering round r         */
+    int64_t a_r[MST_MAX_ROUNDS];          /* alive (local) edge records entering round r's
+                                             pass (dense rounds: matrix entries)          */
     int64_t num_edges;                    /* |F*| of the last run                        */
     uint64_t total_weight;
     double build_ms;                      /* wall time of the build in mst_create*       */
@@ -179,7 +187,8 @@ mst_status mst_set_profiling(mst_graph* g, int enable);
  *       light-edge phase and the pass that then re-reads every record never compact. Never
  *       changes the result.
  *   MST_OPT_LIGHT_FIRST (default -1 = auto; 0 = off, else K in [1, 64]): light-edge phase
- *       (auto: K = 4 when there are >= 64 records per vertex, else K = 2). Kruskal
+ *       (auto: K = 8 with a light-only round 0 when there are >= 64 records per
+ *       vertex, else K = 2; R16). Kruskal
  *       takes the edges in (w, id) order (the "ordered" algorithm), so the
  *       forest restricted to the edges with w <= t is the forest of that light subgraph for
  *       every t. mst_run first picks t so that about K*n edge records are light (a 4096-record
@@ -188,8 +197,12 @@ mst_status mst_set_profiling(mst_graph* g, int enable);
  *       light edge is deferred, not finished — and once no light edge joins two components
  *       re-reads every record (relabelled; all the light ones are now intra-component and
  *       deleted) and continues as usual. Used when at least 4*K*n records exist (dense and
- *       heavy-tailed inputs), on single-GPU handles without MST_OPT_KEEP_EDGES. Never
- *       changes the result.
+ *       heavy-tailed inputs) and MST_OPT_KEEP_EDGES is off, on every kind of handle (a
+ *       distributed run agrees on one t: the minimum of the ranks' sampled thresholds).
+ *       Never changes the result.
+ * Keys of the component minima (rows A2/A8): (uint64(w) << 32) | eid, or, when the largest
+ * weight, the largest edge id and the largest vertex id fit 63 bits together, the packed
+ * (w << s1) | (eid << pb) | partner label — the same (w, eid) order (reading R17).
  */
 enum { MST_OPT_DENSE = 1, MST_OPT_KEEP_EDGES = 2, MST_OPT_DEVICE_TAIL = 3, MST_OPT_COMPACT_TAU = 4,
        MST_OPT_LIGHT_FIRST = 5 };

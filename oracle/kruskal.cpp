@@ -90,7 +90,9 @@ int64_t oracle_kruskal(int64_t n, int64_t m, const int32_t* src, const int32_t* 
 }
 
 // Connected-component labels: label[v] = smallest vertex id in v's component (plain
-// definition of the partition the forest spans; used to pin mst_labels).
+// definition of the partition the forest spans). Its count c gives the forest size n - c
+// that the GPU parity tests check independently of Kruskal (pinned against BFS in
+// tests/test_oracle_pins.py).
 int64_t oracle_components(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                           int32_t* label) {
     for (int64_t i = 0; i < m; ++i)

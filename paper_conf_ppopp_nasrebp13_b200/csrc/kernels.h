@@ -54,13 +54,14 @@ cudaError_t launch_scatter(cudaStream_t st, int nsm, u32 m, const u32* eu, const
 // and fills the unused end of its last block with dead records (owner ~0); *light_count =
 // records written including that filler (<= light + light_blk * warps of the launch)
 cudaError_t launch_min0(cudaStream_t st, int nsm, u64 A, const uint4* arcs, u64* best, u32 nb,
-                        u32* tile_ctrs, u32 seq, uint4* light_out = nullptr,
+                        u32* tile_ctrs, u32& seq, uint4* light_out = nullptr,
                         const u32* light_t = nullptr, u32* light_count = nullptr,
                         u32 light_blk = 0, u32 kfmt = 0);
+// seq: the handle's pass sequence (tile-counter slot parity), consumed only by a launch
 // light_blk | 1 << 31: extract only (no minima; light-only round 0)
 // round-0 minimum over records whose count is on the device (*a_in <= a_max)
 cudaError_t launch_min0_dev(cudaStream_t st, int nsm, const u32* a_in, u64 a_max,
-                            const uint4* arcs, u64* best, u32 nb, u32* tile_ctrs, u32 seq,
+                            const uint4* arcs, u64* best, u32 nb, u32* tile_ctrs, u32& seq,
                             u32 kfmt = 0);
 u32 pass_warps(int nsm);
 unsigned long long kernel_launches();  // kernels launched by this process so far
@@ -85,7 +86,7 @@ cudaError_t launch_jump(cudaStream_t st, int nsm, u32 nr, u32* P, const int* Mtm
 u64 hook_tiles(u64 n);
 cudaError_t launch_filter_min(cudaStream_t st, int nsm, const u32* a_in, u64 a_max,
                               const uint4* in, const int* M, uint4* out, u64* best, u32 nb,
-                              u64* status, u32 epoch, u32* a_next, u32* tile_ctrs, u32 seq,
+                              u64* status, u32 epoch, u32* a_next, u32* tile_ctrs, u32& seq,
                               u64* mat, const CompactCtl& cc = CompactCtl(),
                               const int* hub = nullptr, u32 kfmt = 0);
 // kfmt: key format of the minima the pass emits = s1 | pb << 8 (pb = 0: (w << 32) | eid)

@@ -147,6 +147,8 @@ struct mst_graph {
     u64* trace = nullptr;    // MST_TAIL_TRACE=1 (tools): phase timestamps of the dense tail    // heavy-tailed input: hub row of the dense transition in smem
     int* phi = nullptr;      // composed label map of the records' label space (row A7)
 
+    cudaEvent_t fail_ev = nullptr;  // recorded on the run stream when a run fails: the frees
+                                    // of mst_destroy wait for whatever is still in flight
     bool prof = false;
     std::vector<ProfRec> recs;
     std::vector<cudaEvent_t> evpool;
@@ -186,6 +188,7 @@ void release(mst_graph* g) {
     if (!g) return;
     if (g->comm) ncclCommDestroy(g->comm);
     if (g->cst) {
+        if (g->fail_ev) cudaStreamWaitEvent(g->cst, g->fail_ev, 0);
         for (void* p : g->allocs) cudaFreeAsync(p, g->cst);
         cudaStreamSynchronize(g->cst);
     }
@@ -194,6 +197,7 @@ void release(mst_graph* g) {
     if (g->hmap) cudaFreeHost((void*)g->hmap);
     if (g->trace) cudaFree(g->trace);
     for (auto e : g->evpool) cudaEventDestroy(e);
+    if (g->fail_ev) cudaEventDestroy(g->fail_ev);
     if (g->cst) cudaStreamDestroy(g->cst);
     delete g;
 }
@@ -383,8 +387,8 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CK(cudaMemcpyAsync(g->hcnt + C_WMAX, g->dcnt + C_WMAX, sizeof(u32), cudaMemcpyDeviceToHost,
                        g->cst));
     CK(cudaStreamSynchronize(g->cst));
-    {   // packed minima keys when weight, edge id and a label fit in 63 bits (not with dist,
-        // whose per-round allreduce is format-agnostic anyway; kept simple)
+    {   // packed minima keys when weight, edge id and a label fit in 63 bits (every handle:
+        // the keys' order is the (w, eid) order, so the MIN of a distributed run is unchanged)
         auto bits = [](u64 x) { u32 b = 0; while (x) { ++b; x >>= 1; } return b; };
         const u32 wb = bits(g->hcnt[C_WMAX]), eb = bits(m > 0 ? (u64)m - 1 : 0),
                   pb = bits(n > 0 ? (u64)n - 1 : 0);
@@ -428,6 +432,14 @@ mst_status create_common(int64_t n, int64_t m, const int32_t* src, const int32_t
     if (e != cudaSuccess) {
         release(g);
         return fail(MST_ECUDA, "device setup: %s", cudaGetErrorString(e));
+    }
+    // the inputs may still be written by work in flight on any of the caller's streams (the
+    // build reads them on the handle's own non-blocking stream): wait for the device first
+    // (a one-time cost of the build)
+    if (cudaDeviceSynchronize() != cudaSuccess) {
+        const cudaError_t e2 = cudaGetLastError();
+        release(g);
+        return fail(MST_ECUDA, "device synchronisation before the build: %s", cudaGetErrorString(e2));
     }
     mst_status s = build(g, src, dst, (const unsigned*)w, nshards_sim, rank, nranks, reorder);
     if (s == MST_OK && id != nullptr) {  // mst_create_dist: NCCL communicator (also 1 rank)
@@ -572,15 +584,15 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             const u64 per_warp = (u64)lk * n / ((u64)g->nsm * 30);
             const u32 blk = (u32)std::min<u64>(LBLK_MAX, std::max<u64>(LBLK_MIN, per_warp / 4));
             CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, (u32)n, g->dcnt + C_TILE,
-                           g->pass_seq++, g->abuf[0], g->dcnt + C_LT, g->dcnt + arec(j, 0),
+                           g->pass_seq, g->abuf[0], g->dcnt + C_LT, g->dcnt + arec(j, 0),
                            blk | (light_only0 ? 1u << 31 : 0u), g->kfmt));
             if (light_only0)
                 CK(launch_min0_dev(s, g->nsm, g->dcnt + arec(j, 0),
                                    sh.A + (u64)pass_warps(g->nsm) * LBLK_MAX, g->abuf[0], tgt,
-                                   (u32)n, g->dcnt + C_TILE, g->pass_seq++, g->kfmt));
+                                   (u32)n, g->dcnt + C_TILE, g->pass_seq, g->kfmt));
         } else
             CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, (u32)n, g->dcnt + C_TILE,
-                           g->pass_seq++, nullptr, nullptr, nullptr, 0, g->kfmt));
+                           g->pass_seq, nullptr, nullptr, nullptr, 0, g->kfmt));
     }
     if (g->sim) {
         Prof p(g, s, MST_K_COMM, 0);
@@ -816,7 +828,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                 }
                 CK(launch_filter_min(s, g->nsm, g->dcnt + arec(j, r), sh.hi - sh.lo, cur + sh.lo,
                                      Mpass, out, tgt, nn, g->status, g->epoch++,
-                                     g->dcnt + arec(j, r + 1), g->dcnt + C_TILE, g->pass_seq++,
+                                     g->dcnt + arec(j, r + 1), g->dcnt + C_TILE, g->pass_seq,
                                      to_dense ? g->mat[0] : nullptr, ccj,
                                      (to_dense && use_hub_row(g) && hub_ok)
                                          ? (const int*)g->dcnt + C_HUB + r + 1 : nullptr,
@@ -1050,7 +1062,16 @@ mst_status mst_run(mst_graph* g, mst_stream_t stream, int32_t* out_edge_ids,
         if (!out_num_edges || !out_total_weight) return fail(MST_EINVAL, "null output pointer");
         if (!out_edge_ids && g->n > 1) return fail(MST_EINVAL, "out_edge_ids is NULL");
         mst_status s = run_impl(g, (cudaStream_t)stream, out_edge_ids, out_num_edges, out_total_weight);
-        if (s != MST_OK) g->broken = true;
+        if (s != MST_OK) {
+            g->broken = true;
+            // kernels of the failed run may still be queued or running on `stream`: the
+            // handle's frees are ordered after them (release waits on this event)
+            (void)cudaGetLastError();
+            if (!g->fail_ev && cudaEventCreateWithFlags(&g->fail_ev, cudaEventDisableTiming) != cudaSuccess)
+                g->fail_ev = nullptr;
+            if (g->fail_ev) cudaEventRecord(g->fail_ev, (cudaStream_t)stream);
+            (void)cudaGetLastError();
+        }
         return s;
     });
 }
@@ -1149,7 +1170,7 @@ mst_status mst_debug_filter_pass(mst_graph* g, mst_stream_t stream, int map_kind
             CK(cudaMemsetAsync(g->bestB, 0xff, n * sizeof(u64), s));
             CK(launch_filter_min(s, g->nsm, nullptr, A, g->arcs0 + sh.lo, g->maps,
                                  g->abuf[0] + sh.lo, g->bestB, ncomp, g->status, g->epoch++,
-                                 g->dcnt + arec(0, 1), g->dcnt + C_TILE, g->pass_seq++, nullptr));
+                                 g->dcnt + arec(0, 1), g->dcnt + C_TILE, g->pass_seq, nullptr));
         }
         CK(cudaEventRecord(e1, s));
         CK(cudaEventSynchronize(e1));
