@@ -155,7 +155,20 @@ def min0_byte_model(st):
     written per light record (a_r[0] = the records the pass wrote, incl. the dead filler that
     ends each warp's reserved block)."""
     light = st.get("light_t", 0xFFFFFFFF) != 0xFFFFFFFF
-    return 16 * st["arcs0"] + (16 * st["a_r"][0] if light and st["rounds"] else 0)
+    return 16 * st["local_arcs0"] + (16 * st["a_r"][0] if light and st["rounds"] else 0)
+
+
+def launch_bytes(st, lt, bm):
+    """Algorithmic bytes of one profiled launch: the A2 passes by sub-kind
+    (min_all / extract: every record read + light records written; min_light: the light
+    records read), the A8 passes from the per-round model (bm), anything else 0."""
+    light = st.get("light_t", 0xFFFFFFFF) != 0xFFFFFFFF
+    if lt["kind"] == "min0":
+        wrote = 16 * st["a_r"][0] if light and st["rounds"] else 0
+        return 16 * st["local_arcs0"] + wrote if lt["sub"] in ("min_all", "extract") else wrote
+    if lt["kind"] == "filter" and lt["round"] < len(bm):
+        return bm[lt["round"]]["bytes"]
+    return 0
 
 
 def run_gpu(args):
@@ -189,6 +202,8 @@ def run_gpu(args):
         h.set_option(mstb.mst.MST_OPT_DENSE, 0)
     elif args.mode == "keep":
         h.set_option(mstb.mst.MST_OPT_KEEP_EDGES, 1)
+    elif args.mode == "uf":
+        h.set_option(mstb.mst.MST_OPT_UNION_FIND, 1)
     if args.tau is not None:
         h.set_option(mstb.mst.MST_OPT_COMPACT_TAU, args.tau)
     build_ms = h.stats()["build_ms"]
@@ -228,18 +243,27 @@ def run_gpu(args):
     h.set_profiling(True)
     filt_ms, filt_bytes, filt_launches, prof_ms = 0.0, 0, 0, []
     min0_ms, min0_bytes, min0_launches = 0.0, 0, 0
+    by_kind = {}  # (kind, sub) -> [launches, ms, bytes]: unlike launches kept apart
     round_acc = None
     for _ in range(args.steps):
         (ids, cnt, tot), ms = timed_step()
         prof_ms.append(ms)
         st = h.stats()
-        filt_ms += st["kernel_ms"]["filter"]
-        filt_launches += st["kernel_launches"]["filter"]
         bm = byte_model(st)
-        filt_bytes += sum(x["bytes"] for x in bm if x["kind"] == "filter")
-        min0_ms += st["kernel_ms"]["min0"]
-        min0_launches += st["kernel_launches"]["min0"]
-        min0_bytes += min0_byte_model(st)
+        for lt in h.launch_times():
+            b = launch_bytes(st, lt, bm)
+            acc = by_kind.setdefault((lt["kind"], lt["sub"]), [0, 0.0, 0])
+            acc[0] += 1
+            acc[1] += lt["ms"]
+            acc[2] += b
+            if lt["kind"] == "filter":
+                filt_ms += lt["ms"]
+                filt_launches += 1
+                filt_bytes += b
+            elif lt["kind"] == "min0":
+                min0_ms += lt["ms"]
+                min0_launches += 1
+                min0_bytes += b
         if round_acc is None:
             round_acc = [{"r": r, "kind": bm[r]["kind"], "n_r": st["n_r"][r], "A_r": st["a_r"][r],
                           "compacted": bm[r].get("compacted"),
@@ -335,6 +359,15 @@ def run_gpu(args):
             "roofline_kernels": {
                 "A8 filter": kernel_roof("k_arc_pass<MODE_FILTER> (A8)", filt_ms, filt_bytes, filt_launches),
                 "A2 min0": kernel_roof("k_arc_pass<MODE_MIN0> (A2)", min0_ms, min0_bytes, min0_launches)},
+            # every launch kind on its own (per-launch averages over like launches only)
+            "launch_kinds": {
+                f"{k}/{sb}": {"launches_per_step": v[0] / args.steps,
+                              "ms_per_step": v[1] / args.steps,
+                              "avg_launch_ms": v[1] / v[0],
+                              "bytes_per_launch": v[2] / v[0],
+                              "GBps": (v[2] / (v[1] * 1e-3) / 1e9) if v[1] > 0 and v[2] else None,
+                              "frac": (v[2] / (v[1] * 1e-3) / 1e9 / peak) if v[1] > 0 and v[2] else None}
+                for (k, sb), v in sorted(by_kind.items())},
             "light_phase": {"t": st["light_t"] if st["light_t"] != 0xFFFFFFFF else None,
                             "switch_round": st["light_switch_round"]},
             "rounds": rounds,
@@ -397,9 +430,10 @@ def main():
                     choices=["grid64", "uniform", "road", "rmat22", "dense"])
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--mode", default="morph", choices=["morph", "sparse", "keep"],
+    ap.add_argument("--mode", default="morph", choices=["morph", "sparse", "keep", "uf"],
                     help="morph: delete+compact, dense min-matrix at <= 4096 components "
-                         "(default); sparse: never dense; keep: the paper's no-deletion scheme")
+                         "(default); sparse: never dense; keep: the paper's no-deletion scheme; "
+                         "uf: the union-find variant (NEXT-3)")
     ap.add_argument("--tau", type=int, default=None,
                     help="MST_OPT_COMPACT_TAU (permille; default: the library's)")
     ap.add_argument("--e2e-steps", type=int, default=3)

@@ -127,7 +127,22 @@ enum {
     MST_K_OUTPUT = 5,  /* A11 output compaction                                       */
     MST_K_COMM = 6,    /* A3 cross-GPU MIN (distributed handles)                      */
     MST_K_DENSE = 7,   /* A9 dense rounds over the component min-matrix              */
-    MST_K_COUNT = 8
+    MST_K_LIGHT = 8,   /* A2 light-edge threshold select (sampled radix select)       */
+    MST_K_COMPOSE = 9, /* A7 label-map composition (+ the round-0 survival sample)    */
+    MST_K_COUNT = 10
+};
+/* launch sub-kinds (mst_launch_time.sub), so unlike launches of one kind are told apart:
+ *   MST_K_MIN0  : MIN_ALL   = minima over every record (+ the light-record write);
+ *                 EXTRACT   = light-only round 0: the light-record write alone;
+ *                 MIN_LIGHT = minima over the light records
+ *   MST_K_FILTER: SPARSE = a pass over the alive records; LIGHT = a light-edge phase pass;
+ *                 SWITCH = the pass that re-reads every record after the light phase;
+ *                 TRANSITION = the pass into the dense min-matrix
+ *   MST_K_DENSE : DENSE_ROUND, DENSE_BEST, TAIL (the cooperative device tail) */
+enum {
+    MST_SUB_MIN_ALL = 0, MST_SUB_EXTRACT = 1, MST_SUB_MIN_LIGHT = 2,
+    MST_SUB_SPARSE = 0, MST_SUB_LIGHT = 1, MST_SUB_SWITCH = 2, MST_SUB_TRANSITION = 3,
+    MST_SUB_DENSE_ROUND = 0, MST_SUB_DENSE_BEST = 1, MST_SUB_TAIL = 2
 };
 typedef struct {
     int64_t n, m, arcs0;                  /* vertices, edges, E_0 = #non-loop edges (one
@@ -160,6 +175,16 @@ typedef struct {
 } mst_stats;
 
 mst_status mst_get_stats(const mst_graph* g, mst_stats* out);
+
+/* Per-launch event times of the last PROFILED run (mst_set_profiling), in launch order:
+ * kind (MST_K_*), sub (MST_SUB_*), round, shard (sharded handles), ms. Copies
+ * min(cap, *count) records to out (HOST array); *count = the number of launches recorded. */
+typedef struct {
+    int32_t kind, sub, round, shard;
+    double ms;
+} mst_launch_time;
+mst_status mst_get_launch_times(const mst_graph* g, mst_launch_time* out, int64_t cap,
+                                int64_t* count);
 
 /* enable (1) / disable (0) per-launch CUDA-event timing for subsequent runs */
 mst_status mst_set_profiling(mst_graph* g, int enable);
@@ -200,12 +225,21 @@ mst_status mst_set_profiling(mst_graph* g, int enable);
  *       heavy-tailed inputs) and MST_OPT_KEEP_EDGES is off, on every kind of handle (a
  *       distributed run agrees on one t: the minimum of the ranks' sampled thresholds).
  *       Never changes the result.
+ *   MST_OPT_UNION_FIND (default 0): 1 = the union-find variant (
+ *       PAPER.md §8.4: a component-based Boruvka with a "fast union-find" that "keeps the
+ *       graph unmodified" in a "bulk-synchronous executor"): every round finds both endpoint
+ *       roots of the alive edge records by union-find (path halving), drops intra-component
+ *       records (the survivors are compacted unchanged, never relabelled, under
+ *       MST_OPT_COMPACT_TAU; 0 or MST_OPT_KEEP_EDGES = the unmodified records every round),
+ *       min-reduces per root, and unions the two roots of every chosen edge by CAS. No
+ *       renumbering, no label maps, no dense rounds, no light-edge phase. Single-GPU handles
+ *       only (MST_ENOTSUP from mst_run otherwise). Never changes the result.
  * Keys of the component minima (rows A2/A8): (uint64(w) << 32) | eid, or, when the largest
  * weight, the largest edge id and the largest vertex id fit 63 bits together, the packed
  * (w << s1) | (eid << pb) | partner label — the same (w, eid) order (reading R17).
  */
 enum { MST_OPT_DENSE = 1, MST_OPT_KEEP_EDGES = 2, MST_OPT_DEVICE_TAIL = 3, MST_OPT_COMPACT_TAU = 4,
-       MST_OPT_LIGHT_FIRST = 5 };
+       MST_OPT_LIGHT_FIRST = 5, MST_OPT_UNION_FIND = 6 };
 mst_status mst_set_option(mst_graph* g, int option, int64_t value);
 
 /* ------------------------------------------------------------------ multi-GPU (§8(e))

@@ -30,6 +30,24 @@ mst_status mst_debug_filter_pass(mst_graph* g, mst_stream_t stream, int map_kind
  *                 j * arcs / nranks. Windows are contiguous, disjoint and cover [0, arcs). */
 mst_status mst_shard_ranges(const uint32_t* row_offsets, int64_t n, int nranks, int64_t* lo,
                             int64_t* hi);
+/* mst_create_dist_hostx: a distributed handle (as mst_create_dist) whose
+ * exchange step is a HOST callback instead of NCCL, so that several processes sharing one
+ * GPU (NCCL allows one rank per device) run the real distributed round loop — per-rank
+ * record builds, rank-local compaction decisions, the per-round MIN, the agreed light-edge
+ * threshold — with the MIN done by their own process group (tests: a gloo all_reduce).
+ *   src, dst, w : DEVICE pointers to the identical full input on every rank (as mst_create)
+ *   rank, nranks: this process's rank, the number of ranks (1..64)
+ *   fn          : called by mst_run (on the calling thread, the run's stream synchronised) with
+ *                 a HOST buffer of `count` uint64 words; it must replace every word by the
+ *                 minimum of that word over all ranks (unsigned compare) and return 0, or
+ *                 non-zero to fail the run with MST_ENCCL. Every rank calls it the same
+ *                 number of times with the same counts, in the same order.
+ *   ctx         : passed through to fn.
+ * MST_EINVAL for a NULL fn or bad rank/nranks; otherwise as mst_create_dist. */
+typedef int (*mst_allreduce_min_fn)(uint64_t* host_buf, int64_t count, void* ctx);
+mst_status mst_create_dist_hostx(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
+                                 const uint32_t* w, int rank, int nranks,
+                                 mst_allreduce_min_fn fn, void* ctx, mst_graph** out);
 #ifdef __cplusplus
 }
 #endif

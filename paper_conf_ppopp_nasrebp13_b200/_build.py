@@ -9,7 +9,9 @@ import sys
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
-LIB = os.path.join(PKG, "libmst.so")
+# MST_LIB: load another build of the library (A/B variants built with MST_NVCC_FLAGS into
+# build/ab/; tools/abvar.sh) instead of the in-tree libmst.so
+LIB = os.environ.get("MST_LIB") or os.path.join(PKG, "libmst.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
@@ -37,6 +39,8 @@ def deps():
 
 
 def needs_build() -> bool:
+    if os.environ.get("MST_LIB"):
+        return False  # a prebuilt variant is loaded as it is
     if not os.path.exists(LIB):
         return True
     t = os.path.getmtime(LIB)

@@ -48,7 +48,8 @@ cudaError_t launch_owner_degree(cudaStream_t st, int nsm, u32 m, const u32* eu, 
                                 u32* odeg, int hi_owner);
 cudaError_t launch_scatter(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
                            const unsigned* w, u32* cursor, uint4* arcs, uint2* euv,
-                           int hi_owner, u32* wmax);
+                           int hi_owner, u32* wmax, u32 vlo, u32 vhi, u32 wbase);
+// (only the records of owners in [vlo, vhi), at their CSR position minus wbase)
 // light_out != nullptr (MST_OPT_LIGHT_FIRST): also append the records of weight <= *light_t
 // to light_out; every consumer warp reserves blocks of light_blk records (one atomic each)
 // and fills the unused end of its last block with dead records (owner ~0); *light_count =
@@ -63,11 +64,12 @@ cudaError_t launch_min0(cudaStream_t st, int nsm, u64 A, const uint4* arcs, u64*
 cudaError_t launch_min0_dev(cudaStream_t st, int nsm, const u32* a_in, u64 a_max,
                             const uint4* arcs, u64* best, u32 nb, u32* tile_ctrs, u32& seq,
                             u32 kfmt = 0);
-u32 pass_warps(int nsm);
+u32 pass_warps(int nsm);  // consumer warps of one pass launch, rounded up (the filler bound)
 unsigned long long kernel_launches();  // kernels launched by this process so far
-// A1: best = inf (n), msf = 0 (nwords), acc = 0 (nacc), ctr = 0 (nctr), *zero1 = *zero2 = 0
+// A1: best = inf (n), msf = 0 (nwords), acc = 0 (nacc), ctr = 0 (nctr), *zero1 = 0,
+// ctr2 = 0 (nctr2: every per-shard, per-round record count of the run)
 cudaError_t launch_init(cudaStream_t st, int nsm, u32 n, u64* best, u32 nwords, u32* msf,
-                        u64* acc, u32 nacc, u32* ctr, u32 nctr, u32* zero1, u32* zero2);  // consumer warps of one pass launch (the filler bound)
+                        u64* acc, u32 nacc, u32* ctr, u32 nctr, u32* zero1, u32* ctr2, u32 nctr2);
 // weight threshold t of the light-edge phase: about `target` of the A records have w <= t
 // (binary search on a 4096-record sample); writes *t
 cudaError_t launch_light_threshold(cudaStream_t st, const uint4* arcs, u64 A, u64 target, u32* t);
@@ -89,6 +91,18 @@ cudaError_t launch_filter_min(cudaStream_t st, int nsm, const u32* a_in, u64 a_m
                               u64* status, u32 epoch, u32* a_next, u32* tile_ctrs, u32& seq,
                               u64* mat, const CompactCtl& cc = CompactCtl(),
                               const int* hub = nullptr, u32 kfmt = 0);
+// NEXT-3 union-find variant: parent = identity; one pass (K1: roots by find,
+// intra-component records dropped, survivors compacted unchanged when the policy says so,
+// minima keys (w << s1 | eid) | tag into best[root]); then partner + union (K2a/K2b: forest
+// bits, forest weight/size into acc, *unions += unions; K2a first publishes *surv to hmap)
+cudaError_t launch_uf_init(cudaStream_t st, int nsm, u32 n, u32* parent);
+cudaError_t launch_uf_pass(cudaStream_t st, int nsm, const u32* a_in, u64 a_max, const uint4* in,
+                           u32* parent, uint4* out, u64* best, u32 n, u64* status, u32 epoch,
+                           u32* a_next, u32* tile_ctrs, u32& seq, const CompactCtl& cc, u32 s1,
+                           u64 tag);
+cudaError_t launch_uf_hook(cudaStream_t st, int nsm, u32 n, u32* parent, const u64* best, u32 s1,
+                           bool tagged, u64 tag, const uint2* euv, u32* P, u32* msf, u64* acc,
+                           u32* unions, const u32* surv, u64* hmap, u32 htag);
 // kfmt: key format of the minima the pass emits = s1 | pb << 8 (pb = 0: (w << 32) | eid)
 cudaError_t launch_dense_best(cudaStream_t st, int nsm, u32 n, const u64* mat, u64* best);
 cudaError_t launch_dense_init(cudaStream_t st, int nsm, u32 n, u64* mat);

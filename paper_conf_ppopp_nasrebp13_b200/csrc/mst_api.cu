@@ -87,16 +87,24 @@ constexpr int C_LT = C_HUB + MST_MAX_ROUNDS + 1;  // light-edge threshold t
 constexpr int C_WMAX = C_LT + 1;                   // largest weight (build)
 constexpr int C_TAILN = C_WMAX + 1;                // light-phase tail: labels after it
 constexpr u32 LBLK_MIN = 32, LBLK_MAX = 256;      // light write: records per warp reservation
-constexpr int DCNT_WORDS = C_TAILN + 1;
+constexpr int C_UFU = C_TAILN + 1;                 // union-find variant: unions per round
+constexpr int DCNT_WORDS = C_UFU + MST_MAX_ROUNDS;
 constexpr int HSURV = MST_MAX_ROUNDS + 1;  // mapped words: [0, HSURV) sizes, [HSURV, 2 HSURV) decisions
 
 struct Shard {
-    u64 lo, hi;  // arc range [lo, hi) in arcs_0 and in the ping-pong buffers
-    u32 A;       // alive arcs entering the current round
+    u64 lo, hi;  // record window [lo, hi) in the handle's arcs0 and in the ping-pong buffers
+    u64 llo;     // window start of the shard's light records in abuf[0] (light-edge phase):
+                 // lo + j * light slack, so every shard has room for its filler records
+    u32 A;       // alive records entering the current round
 };
 
+// Exchange of a distributed handle (row A3): NCCL over NVLink in production; a host callback
+// (mst_create_dist_hostx, test aid) lets several processes that share one GPU run the same
+// round loop with the MIN done by their own process group.
+enum XKind { X_NONE = 0, X_NCCL = 1, X_HOST = 2 };
+
 struct ProfRec {
-    int kind, round;
+    int kind, round, sub, shard;
     cudaEvent_t a, b;
 };
 
@@ -136,7 +144,14 @@ struct mst_graph {
     bool sim = false;
     int rank = 0, nranks = 1;
     ncclComm_t comm = nullptr;
+    int xkind = X_NONE;
+    mst_allreduce_min_fn xfn = nullptr;  // X_HOST: allreduce-MIN of u64 in host memory
+    void* xctx = nullptr;
+    u64* xhost = nullptr;                // X_HOST: pinned staging (n + dense matrix entries)
+    u64 xcap = 0;
+    u64 A0_local = 0;                    // records built on this rank (all shards)
 
+    bool opt_uf = false;     // MST_OPT_UNION_FIND (NEXT-3 variant)
     bool opt_dense = true;   // MST_OPT_DENSE
     bool opt_keep = false;   // MST_OPT_KEEP_EDGES (paper-faithful ablation)
     bool opt_tail = true;    // MST_OPT_DEVICE_TAIL
@@ -151,6 +166,7 @@ struct mst_graph {
                                     // of mst_destroy wait for whatever is still in flight
     bool prof = false;
     std::vector<ProfRec> recs;
+    std::vector<mst_launch_time> ltimes;  // per launch of the last profiled run
     std::vector<cudaEvent_t> evpool;
     size_t evused = 0;
     mst_stats st{};
@@ -195,6 +211,7 @@ void release(mst_graph* g) {
     if (g->hcnt) cudaFreeHost(g->hcnt);
     if (g->hacc) cudaFreeHost(g->hacc);
     if (g->hmap) cudaFreeHost((void*)g->hmap);
+    if (g->xhost) cudaFreeHost(g->xhost);
     if (g->trace) cudaFree(g->trace);
     for (auto e : g->evpool) cudaEventDestroy(e);
     if (g->fail_ev) cudaEventDestroy(g->fail_ev);
@@ -215,10 +232,10 @@ cudaEvent_t next_event(mst_graph* g) {
 struct Prof {
     mst_graph* g;
     cudaStream_t s;
-    int kind, round;
+    int kind, round, sub, shard;
     cudaEvent_t a = nullptr;
-    Prof(mst_graph* g_, cudaStream_t s_, int kind_, int round_)
-        : g(g_), s(s_), kind(kind_), round(round_) {
+    Prof(mst_graph* g_, cudaStream_t s_, int kind_, int round_, int sub_ = 0, int shard_ = 0)
+        : g(g_), s(s_), kind(kind_), round(round_), sub(sub_), shard(shard_) {
         if (g->prof) {
             a = next_event(g);
             cudaEventRecord(a, s);
@@ -228,7 +245,7 @@ struct Prof {
         if (g->prof) {
             cudaEvent_t b = next_event(g);
             cudaEventRecord(b, s);
-            g->recs.push_back({kind, round, a, b});
+            g->recs.push_back({kind, round, sub, shard, a, b});
         }
     }
 };
@@ -245,7 +262,7 @@ mst_status check_args(int64_t n, int64_t m, const void* src, const void* dst, co
 // Arc-balanced source ranges: shard j owns the sources [v_j, v_{j+1}),
 // v_j = the first vertex whose CSR row offset reaches j * A0 / G; returns the arc windows
 // [row[v_j], row[v_{j+1}]). Pure host code (exported for tests as mst_shard_ranges).
-void compute_shard_ranges(const u32* row, u64 n, int G, u64* lo, u64* hi) {
+void compute_shard_ranges(const u32* row, u64 n, int G, u64* lo, u64* hi, u64* vbo = nullptr) {
     const u64 A0 = row[n];
     std::vector<u64> vb(G + 1);
     vb[0] = 0;
@@ -259,11 +276,16 @@ void compute_shard_ranges(const u32* row, u64 n, int G, u64* lo, u64* hi) {
         lo[j] = row[vb[j]];
         hi[j] = row[vb[j + 1]];
     }
+    if (vbo)
+        for (int j = 0; j <= G; ++j) vbo[j] = vb[j];
 }
 
-mst_status shard_ranges(mst_graph* g, int G, std::vector<u64>& lo, std::vector<u64>& hi) {
+mst_status shard_ranges(mst_graph* g, int G, std::vector<u64>& lo, std::vector<u64>& hi,
+                        std::vector<u64>& vb) {
     lo.assign(G, 0);
     hi.assign(G, 0);
+    vb.assign(G + 1, 0);
+    vb[G] = (u64)g->n;
     if (G == 1) {
         hi[0] = g->A0;
         return MST_OK;
@@ -272,7 +294,7 @@ mst_status shard_ranges(mst_graph* g, int G, std::vector<u64>& lo, std::vector<u
     CK(cudaMemcpyAsync(row.data(), g->row, (g->n + 1) * sizeof(u32), cudaMemcpyDeviceToHost,
                        g->cst));
     CK(cudaStreamSynchronize(g->cst));
-    compute_shard_ranges(row.data(), g->n, G, lo.data(), hi.data());
+    compute_shard_ranges(row.data(), g->n, G, lo.data(), hi.data(), vb.data());
     return MST_OK;
 }
 
@@ -347,28 +369,37 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     u32 A0;
     CK(cudaMemcpyAsync(&A0, g->row + n, sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
     CK(cudaStreamSynchronize(g->cst));
-    g->A0 = A0;
-    CKS(galloc(g, &g->arcs0, A0));
+    g->A0 = A0;  // every rank's records together (the global E_0: identical decisions)
+
+    // shards: owner-vertex ranges balanced by records. The simulation keeps
+    // all G ranges in one handle; a distributed rank builds ONLY the records of its own range
+    const int G = nshards_sim > 1 ? nshards_sim : nranks;
+    std::vector<u64> lo, hi, vb;
+    CKS(shard_ranges(g, G, lo, hi, vb));
+    u64 wbase = 0, vlo = 0, vhi = n;  // the records this handle builds: owners [vlo, vhi)
+    if (nshards_sim <= 1 && G > 1) {
+        wbase = lo[rank];
+        vlo = vb[rank];
+        vhi = vb[rank + 1];
+    }
+    const u64 A_loc = (nshards_sim <= 1 && G > 1) ? hi[rank] - lo[rank] : (u64)A0;
+    g->A0_local = A_loc;
+    CKS(galloc(g, &g->arcs0, A_loc));
     CKS(galloc(g, &g->euv, m));
     CK(launch_scatter(g->cst, g->nsm, (u32)m, g->eu, g->ev, w, cursor, g->arcs0, g->euv, hi_owner,
-                      g->dcnt + C_WMAX));
-
-    // shards: simulation = all G ranges locally; distributed = this rank's range only
-    const int G = nshards_sim > 1 ? nshards_sim : nranks;
-    std::vector<u64> lo, hi;
-    CKS(shard_ranges(g, G, lo, hi));
+                      g->dcnt + C_WMAX, (u32)vlo, (u32)vhi, (u32)wbase));
     g->shards.clear();
-    u64 cap = 0;
+    // light-edge phase: each shard's light records and their dead filler records (at most
+    // LBLK_MAX per consumer warp of the pass) get their own window in abuf[0]
+    const u64 slack = (u64)pass_warps(g->nsm) * LBLK_MAX;
     for (int j = 0; j < G; ++j) {
         if (nshards_sim <= 1 && j != rank) continue;
-        g->shards.push_back({lo[j], hi[j], (u32)(hi[j] - lo[j])});
-        cap = std::max(cap, hi[j]);
+        const u64 l = lo[j] - wbase, h = hi[j] - wbase, k = g->shards.size();
+        g->shards.push_back({l, h, l + k * slack, (u32)(h - l)});
     }
-    // ping-pong arc buffers: a shard's arcs keep their [lo, hi) window in every buffer
-    // abuf[0] also takes the light-edge write of a single-GPU handle: the light records plus
-    // at most LBLK_MAX dead filler records per consumer warp (MST_OPT_LIGHT_FIRST)
-    for (int b = 0; b < 2; ++b)
-        CKS(galloc(g, &g->abuf[b], cap + (b == 0 && G == 1 ? (u64)pass_warps(g->nsm) * LBLK_MAX : 0)));
+    // ping-pong record buffers: a shard's records keep their [lo, hi) window in every buffer
+    CKS(galloc(g, &g->abuf[0], A_loc + g->shards.size() * slack));
+    CKS(galloc(g, &g->abuf[1], A_loc));
     CKS(galloc(g, &g->bestA, n));
     CKS(galloc(g, &g->bestB, n));
     if (g->sim) CKS(galloc(g, &g->shard_best, n * (u64)g->shards.size()));
@@ -400,9 +431,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     g->st.arcs0 = (int64_t)g->A0;
     g->st.nranks = nranks;
     g->st.rank = rank;
-    u64 local = 0;
-    for (auto& s : g->shards) local += s.hi - s.lo;
-    g->st.local_arcs0 = (int64_t)local;
+    g->st.local_arcs0 = (int64_t)g->A0_local;
     g->st.build_ms =
         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     return MST_OK;
@@ -410,7 +439,8 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
 
 mst_status create_common(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                          const uint32_t* w, int nshards_sim, const uint8_t* id, int rank,
-                         int nranks, mst_graph** out, bool reorder = true) {
+                         int nranks, mst_graph** out, bool reorder = true,
+                         mst_allreduce_min_fn xfn = nullptr, void* xctx = nullptr) {
     if (!out) return fail(MST_EINVAL, "out is NULL");
     *out = nullptr;
     CKS(check_args(n, m, src, dst, w));
@@ -447,6 +477,18 @@ mst_status create_common(int64_t n, int64_t m, const int32_t* src, const int32_t
         memcpy(&uid, id, sizeof uid);
         ncclResult_t r = ncclCommInitRank(&g->comm, nranks, uid, rank);
         if (r != ncclSuccess) s = fail(MST_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
+        else g->xkind = X_NCCL;
+    }
+    if (s == MST_OK && xfn != nullptr) {  // host-callback exchange (test aid)
+        g->xkind = X_HOST;
+        g->xfn = xfn;
+        g->xctx = xctx;
+        g->xcap = std::max<u64>((u64)n, dense_entries((u64)n)) + 1;
+        const cudaError_t e2 = cudaMallocHost(&g->xhost, g->xcap * sizeof(u64));
+        if (e2 != cudaSuccess) {
+            g->xhost = nullptr;
+            s = fail(MST_ENOMEM, "pinned exchange staging: %s", cudaGetErrorString(e2));
+        }
     }
     if (s != MST_OK) {
         std::string keep = g_err;
@@ -493,10 +535,180 @@ mst_status wait_round(mst_graph* g, cudaStream_t s, int r, u32 tag, u32* nn) {
     return wait_word(g, s, r, tag, nn);
 }
 
+// A3: allreduce-MIN over the ranks of a distributed handle, in place on the device (u64
+// minima keys, or u32 for the light-edge threshold). NCCL: one ncclAllReduce on the run's
+// stream. Host exchange (test aid): device -> pinned host, the caller's callback reduces across
+// its processes, host -> device; the stream is synchronised around it.
+mst_status xchg_min(mst_graph* g, cudaStream_t s, void* buf, u64 count, bool u32w) {
+    if (count == 0 || g->xkind == X_NONE) return MST_OK;
+    if (g->xkind == X_NCCL) {
+        CKN(ncclAllReduce(buf, buf, count, u32w ? ncclUint32 : ncclUint64, ncclMin, g->comm, s));
+        return MST_OK;
+    }
+    if (count > g->xcap) return fail(MST_EINTERNAL, "exchange of %llu words > staging", (unsigned long long)count);
+    const size_t es = u32w ? 4 : 8;
+    CK(cudaMemcpyAsync(g->xhost, buf, count * es, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    u32* x32 = reinterpret_cast<u32*>(g->xhost);
+    if (u32w)  // widen in place (downwards: entry i is read before bytes [8i, 8i + 8) are written)
+        for (u64 i = count; i-- > 0;) g->xhost[i] = (u64)x32[i];
+    if (g->xfn(g->xhost, (int64_t)count, g->xctx) != 0)
+        return fail(MST_ENCCL, "host exchange callback failed (rank %d)", g->rank);
+    if (u32w)
+        for (u64 i = 0; i < count; ++i) x32[i] = (u32)g->xhost[i];
+    CK(cudaMemcpyAsync(buf, g->xhost, count * es, cudaMemcpyHostToDevice, s));
+    CK(cudaStreamSynchronize(s));
+    return MST_OK;
+}
+
 bool use_hub_row(const mst_graph* g) {
     static const char* e = getenv("MST_HUB_ROW");  // "0" / "1": override (ablation)
     if (e && (e[0] == '0' || e[0] == '1')) return e[0] == '1';
     return g->hub_row;
+}
+
+// per-launch event times of a profiled run -> kernel_ms / kernel_launches / round times
+void collect_profile(mst_graph* g) {
+    g->ltimes.clear();
+    if (g->prof) {
+        for (auto& rc : g->recs) {
+            float ms = 0;
+            cudaEventElapsedTime(&ms, rc.a, rc.b);
+            g->ltimes.push_back({rc.kind, rc.sub, rc.round, rc.shard, (double)ms});
+            g->st.kernel_ms[rc.kind] += ms;
+            g->st.kernel_launches[rc.kind] += 1;
+            if ((rc.kind == MST_K_FILTER || rc.kind == MST_K_DENSE) && rc.round < MST_MAX_ROUNDS)
+                g->st.round_filter_ms[rc.round] += ms;
+        }
+    }
+    g->st.profiling = g->prof ? 1 : 0;
+}
+
+// ---------------------------------------------------------------- NEXT-3: union-find variant
+// Bulk-synchronous Boruvka over the unmodified edge records with a union-find (§8.4
+// L389; kernels in kernels.cu "NEXT-3"). Per round r: K1 = k_arc_pass<MODE_UF>
+// (roots by find, intra-component records dropped, survivors compacted unchanged when the
+// policy says so, tagged minima into best[root]); K2a/K2b = partner roots, then forest bits
+// and CAS unions. One host round trip per round: K1's survivor count (zero: done).
+mst_status run_uf(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out_num,
+                  uint64_t* out_total, unsigned long long kl0) {
+    const u64 n = g->n;
+    if (g->shards.size() != 1 || g->xkind != X_NONE)
+        return fail(MST_ENOTSUP, "MST_OPT_UNION_FIND: single-GPU handles only");
+    Shard& sh = g->shards[0];
+    u32* parent = reinterpret_cast<u32*>(g->Mtmp);  // (the morph path's scratch, n words)
+    {
+        Prof p(g, s, MST_K_INIT, 0);
+        CK(launch_init(s, g->nsm, (u32)n, g->bestA, (u32)std::max<u64>(g->nwords, 1), g->msf,
+                       g->acc, 2 * ACC_SLOTS, g->dcnt + C_SEEN, 2 * MST_MAX_ROUNDS,
+                       g->dcnt + C_UFU, g->dcnt + C_AREC, AREC_STRIDE));
+        CK(launch_uf_init(s, g->nsm, (u32)n, parent));
+        CK(cudaMemsetAsync(g->dcnt + C_UFU, 0, MST_MAX_ROUNDS * sizeof(u32), s));
+    }
+    // key format: tagged when weight and edge-id bits fit below the 6-bit round tag
+    auto bits = [](u64 x) { u32 b = 0; while (x) { ++b; x >>= 1; } return b; };
+    const u32 wb = bits(g->hcnt[C_WMAX]), eb = bits(g->m > 0 ? (u64)g->m - 1 : 0);
+    static const char* te = getenv("MST_UF_TAG");  // "0": untagged keys + a reset per round
+    const bool tagged = wb + eb <= 58 && !(te && te[0] == '0');
+    const u32 s1 = tagged ? eb : 32u;
+    g->hcnt[arec(0, 0)] = sh.A = (u32)(sh.hi - sh.lo);
+    CK(cudaMemcpyAsync(g->dcnt + arec(0, 0), g->hcnt + arec(0, 0), sizeof(u32),
+                       cudaMemcpyHostToDevice, s));
+    const u32 tag_base = ((++g->run_seq) & 0xffffffu) << 8;
+    const uint4* cur = g->arcs0;
+    g->st.compacted_mask = 0;
+    g->st.dense_round = -1;
+    g->st.light_switch_round = -1;
+    g->st.light_t = 0xffffffffu;
+    g->st.hub_row = 0;
+    for (int i = 0; i < MST_MAX_ROUNDS; ++i) g->st.survival_permille[i] = -1;
+    int r = 0;
+    while (true) {
+        if (r >= 63) return fail(MST_EINTERNAL, "union-find variant: round limit exceeded");
+        const u64 tag = tagged ? (u64)(62 - r) << 58 : 0ull;
+        if (!tagged && r > 0) CK(cudaMemsetAsync(g->bestA, 0xff, n * sizeof(u64), s));
+        // compaction of the survivors (unchanged records): never in round 0 (every non-loop
+        // record crosses two singletons), else as the morph passes (MST_OPT_COMPACT_TAU)
+        const bool never = r == 0 || g->tau == 0 || g->opt_keep;
+        const bool adaptive = !never && g->tau < 1000;
+        const uint4* outbuf = (cur == g->abuf[0]) ? g->abuf[1] : g->abuf[0];
+        CompactCtl cc;
+        cc.surv = g->dcnt + C_SURV + r;
+        cc.seen = g->dcnt + C_SEEN + r;
+        if (adaptive) {
+            cc.tau = g->tau;
+            cc.num = g->dcnt + C_SURV + (r - 1);
+            cc.den = g->dcnt + C_SEEN + (r - 1);
+            cc.hword = g->dmap + HSURV + r;
+            cc.tag = tag_base | (u32)r;
+        }
+        {
+            Prof p(g, s, MST_K_FILTER, r, MST_SUB_SPARSE);
+            CK(launch_uf_pass(s, g->nsm, g->dcnt + arec(0, r), sh.hi - sh.lo, cur, parent,
+                              never ? nullptr : const_cast<uint4*>(outbuf), g->bestA, (u32)n,
+                              g->status, g->epoch++, g->dcnt + arec(0, r + 1), g->dcnt + C_TILE,
+                              g->pass_seq, cc, s1, tag));
+        }
+        {
+            Prof p(g, s, MST_K_HOOK, r);
+            CK(launch_uf_hook(s, g->nsm, (u32)n, parent, g->bestA, s1, tagged, tag, g->euv, g->P,
+                              g->msf, g->acc, g->dcnt + C_UFU + r, g->dcnt + C_SURV + r,
+                              g->dmap + r, tag_base | (u32)r));
+        }
+        u32 surv;
+        CKS(wait_round(g, s, r, tag_base | (u32)r, &surv));
+        if (!never) {
+            u32 word = 1;  // (always compacting: tau >= 1000)
+            if (adaptive) {
+                CKS(wait_word(g, s, HSURV + r, tag_base | (u32)r, &word));
+                g->st.survival_permille[r] = (int32_t)(word >> 1);
+            }
+            if (word & 1u) {
+                cur = outbuf;
+                g->st.compacted_mask |= 1ll << r;
+            }
+        }
+        ++r;
+        if (surv == 0) break;  // no record joins two components: the forest is complete
+    }
+    g->st.rounds = r;
+    CK(cudaMemcpyAsync(g->hcnt + C_AREC, g->dcnt + C_AREC, AREC_STRIDE * sizeof(u32),
+                       cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(g->hcnt + C_UFU, g->dcnt + C_UFU, MST_MAX_ROUNDS * sizeof(u32),
+                       cudaMemcpyDeviceToHost, s));
+    {
+        Prof p(g, s, MST_K_OUTPUT, r);
+        if (g->nwords) {
+            CK(launch_output(s, (u32)g->nwords, g->msf, out_ids, g->tcnt, g->dcnt + C_OUT,
+                             (u32)std::max<int64_t>(n - 1, 1)));
+        } else {
+            CK(cudaMemsetAsync(g->dcnt + C_OUT, 0, sizeof(u32), s));
+        }
+    }
+    CK(cudaMemcpyAsync(g->hcnt, g->dcnt, 2 * sizeof(u32), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(g->hacc, g->acc, 2 * ACC_SLOTS * sizeof(u64), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    for (int i = 1; i < ACC_SLOTS; ++i) {
+        g->hacc[0] += g->hacc[2 * i];
+        g->hacc[1] += g->hacc[2 * i + 1];
+    }
+    int64_t comps = (int64_t)n;  // components (incl. isolated vertices) entering each round
+    for (int rr = 0; rr < r; ++rr) {
+        g->st.n_r[rr] = comps;
+        g->st.a_r[rr] = g->hcnt[arec(0, rr)];
+        comps -= g->hcnt[C_UFU + rr];
+    }
+    if ((u64)g->hcnt[C_OUT] != g->hacc[1])
+        return fail(MST_EINTERNAL, "forest size mismatch: %u ids vs %llu unions", g->hcnt[C_OUT],
+                    (unsigned long long)g->hacc[1]);
+    if (g->hacc[1] >= n) return fail(MST_EINTERNAL, "forest has >= n edges");
+    *out_num = (int64_t)g->hacc[1];
+    *out_total = g->hacc[0];
+    g->st.num_edges = *out_num;
+    g->st.total_weight = *out_total;
+    collect_profile(g);
+    g->st.gpu_launches = (int64_t)(kernel_launches() - kl0);
+    return MST_OK;
 }
 
 mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out_num,
@@ -522,16 +734,18 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         g->st.total_weight = 0;
         return MST_OK;
     }
+    if (g->opt_uf) return run_uf(g, s, out_ids, out_num, out_total, kl0);
     const int G = (int)g->shards.size();
     // ---- A1 init
     {
         Prof p(g, s, MST_K_INIT, 0);
         // best_0 = inf, forest bits, accumulators, per-pass counters (C_SEEN, C_SURV), the
-        // hub label (round 0: vertex 0 itself) and shard 0's round-0 record count
+        // hub label (round 0: vertex 0 itself) and every shard's per-round record counts (a
+        // pass that meets no record must not read a count an earlier run left)
         static_assert(C_SURV == C_SEEN + MST_MAX_ROUNDS, "counter layout");
         CK(launch_init(s, g->nsm, (u32)n, g->bestA, (u32)std::max<u64>(g->nwords, 1), g->msf,
                        g->acc, 2 * ACC_SLOTS, g->dcnt + C_SEEN, 2 * MST_MAX_ROUNDS,
-                       g->dcnt + C_HUB, g->dcnt + arec(0, 0)));
+                       g->dcnt + C_HUB, g->dcnt + C_AREC, (u32)G * AREC_STRIDE));
         if (g->sim) CK(cudaMemsetAsync(g->shard_best, 0xff, n * G * sizeof(u64), s));
     }
     // light-edge phase (MST_OPT_LIGHT_FIRST): single handle, enough records to pay
@@ -549,13 +763,15 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     const bool lo0_want = lo_env ? lo_env[0] == '1' : (g->light_k < 0 && dense_regime);
     const u32 lk = lk_env != 0xffffffffu ? lk_env
                  : g->light_k >= 0 ? (u32)g->light_k : (lo0_want ? 8u : 2u);
-    int phase = (lk > 0 && G == 1 && !g->comm && !g->opt_keep && g->A0 >= 4096 &&
+    // (decided on the global record count E_0: every rank of a distributed run agrees)
+    int phase = (lk > 0 && !g->opt_keep && g->A0 >= 4096 &&
                  g->A0 >= 4ull * lk * n) ? 1 : 0;  // light records <= a quarter
+    const bool dist = g->xkind != X_NONE;
     const bool light_only0 = lo0_want && phase;
     g->st.light_switch_round = -1;
     g->st.light_t = 0xffffffffu;
     if (phase) {
-        Prof p(g, s, MST_K_MIN0, 0);
+        Prof p(g, s, MST_K_LIGHT, 0);
         static const char* tf = getenv("MST_LIGHT_T");  // ablation: a fixed threshold
         if (tf) {
             g->hcnt[C_LT] = (u32)strtoul(tf, nullptr, 10);
@@ -568,7 +784,19 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             // vertices without a light edge and one more all-records pass — stays unlikely)
             const bool auto_k = lk_env == 0xffffffffu && g->light_k < 0;
             const u64 target = !auto_k ? (u64)lk * n : lo0_want ? (u64)10 * n : (u64)23 * n / 10;
-            CK(launch_light_threshold(s, g->arcs0, g->A0, target, g->dcnt + C_LT));
+            // a rank samples its own records, aimed at the same fraction of them; every rank
+            // must use the SAME t (a mixed threshold is not a prefix of the (w, id) order),
+            // so the ranks agree on the smallest sampled t
+            const u64 Al = g->A0_local;
+            if (Al == 0)
+                CK(cudaMemsetAsync(g->dcnt + C_LT, 0xff, sizeof(u32), s));
+            else
+                CK(launch_light_threshold(s, g->arcs0, Al, (u64)((double)target * Al / g->A0),
+                                          g->dcnt + C_LT));
+        }
+        if (dist) {
+            Prof p(g, s, MST_K_COMM, 0);
+            CKS(xchg_min(g, s, g->dcnt + C_LT, 1, true));
         }
     }
     // ---- A2 round-0 minimum (+ A3); with the light phase it also writes the light records
@@ -577,29 +805,38 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         sh.A = (u32)(sh.hi - sh.lo);
         u64* tgt = g->sim ? g->shard_best + (u64)j * n : g->bestA;
         if (sh.A == 0) continue;
-        Prof p(g, s, MST_K_MIN0, 0);
         if (phase) {
             // a quarter of a warp's expected light records per reservation: few atomics on
-            // the counter, filler <= a quarter of them
-            const u64 per_warp = (u64)lk * n / ((u64)g->nsm * 30);
+            // the counter, filler <= a quarter of them (the shard's share of ~K n records)
+            const u64 per_warp = (u64)((double)lk * n * sh.A / g->A0) / ((u64)g->nsm * 30);
             const u32 blk = (u32)std::min<u64>(LBLK_MAX, std::max<u64>(LBLK_MIN, per_warp / 4));
-            CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, (u32)n, g->dcnt + C_TILE,
-                           g->pass_seq, g->abuf[0], g->dcnt + C_LT, g->dcnt + arec(j, 0),
-                           blk | (light_only0 ? 1u << 31 : 0u), g->kfmt));
-            if (light_only0)
+            {
+                Prof p(g, s, MST_K_MIN0, 0, light_only0 ? MST_SUB_EXTRACT : MST_SUB_MIN_ALL, j);
+                CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, (u32)n, g->dcnt + C_TILE,
+                               g->pass_seq, g->abuf[0] + sh.llo, g->dcnt + C_LT,
+                               g->dcnt + arec(j, 0), blk | (light_only0 ? 1u << 31 : 0u), g->kfmt));
+            }
+            if (light_only0) {
+                Prof p(g, s, MST_K_MIN0, 0, MST_SUB_MIN_LIGHT, j);
                 CK(launch_min0_dev(s, g->nsm, g->dcnt + arec(j, 0),
-                                   sh.A + (u64)pass_warps(g->nsm) * LBLK_MAX, g->abuf[0], tgt,
-                                   (u32)n, g->dcnt + C_TILE, g->pass_seq, g->kfmt));
-        } else
+                                   sh.A + (u64)pass_warps(g->nsm) * LBLK_MAX, g->abuf[0] + sh.llo,
+                                   tgt, (u32)n, g->dcnt + C_TILE, g->pass_seq, g->kfmt));
+            }
+        } else {
+            Prof p(g, s, MST_K_MIN0, 0, MST_SUB_MIN_ALL, j);
             CK(launch_min0(s, g->nsm, sh.A, g->arcs0 + sh.lo, tgt, (u32)n, g->dcnt + C_TILE,
                            g->pass_seq, nullptr, nullptr, nullptr, 0, g->kfmt));
+        }
     }
     if (g->sim) {
         Prof p(g, s, MST_K_COMM, 0);
         CK(launch_combine_min(s, g->nsm, (u32)n, G, g->shard_best, n, g->bestA));
-    } else if (g->comm) {
+    } else if (dist) {
+        // edge-once records: a vertex's round-0 minimum has contributions from every rank
+        // that owns one of its edges (the other endpoint's side), so round 0 needs a
+        // reduction too, not an allgather of rank-local minima
         Prof p(g, s, MST_K_COMM, 0);
-        CKN(ncclAllReduce(g->bestA, g->bestA, n, ncclUint64, ncclMin, g->comm, s));
+        CKS(xchg_min(g, s, g->bestA, n, false));
     }
 
     // round-0 arc counts (host-known) into the per-round record
@@ -619,6 +856,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     // (n_b = nb_sz labels); a pass whose compaction was decided on the device (sampled) is
     // resolved at the next round's wait (pend)
     const uint4* cur = phase ? g->abuf[0] : g->arcs0;  // light phase: the light records
+    bool cur_light = phase != 0;  // cur holds light records at the shards' llo windows
+    auto off = [&](const Shard& sh) { return cur_light ? sh.llo : sh.lo; };
     int brnd = 0;
     u32 nb_sz = (u32)n;
     int pend = -1;
@@ -630,6 +869,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         g->st.survival_permille[pend] = (int32_t)(word >> 1);  // the estimate the pass used
         if (word & 1u) {
             cur = pend_out;
+            cur_light = false;
             brnd = pend + 1;
             nb_sz = (u32)g->st.n_r[pend + 1];
             g->st.compacted_mask |= 1ll << pend;
@@ -649,7 +889,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             return fail(MST_EINTERNAL, "round limit exceeded (r = %d)", r);
         if (dense && g->opt_tail) {
             // every remaining round in one cooperative launch (A4/A5/A6/A9 on the device)
-            Prof p(g, s, MST_K_DENSE, r);
+            Prof p(g, s, MST_K_DENSE, r, MST_SUB_TAIL);
             static const bool tr = getenv("MST_TAIL_TRACE") && getenv("MST_TAIL_TRACE")[0] == '1';
             if (tr && !g->trace) {
                 CK(cudaMalloc(&g->trace, 64 * sizeof(u64)));
@@ -747,24 +987,27 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             dense = false;  // the records are read again (a dense phase-1 matrix is dropped)
             g->st.light_switch_round = r;
             if (r >= 1 && chain.len + 1 < MST_CHAIN_MAX) {  // Ψ = Mr ∘ chain in one kernel
-                Prof p(g, s, MST_K_JUMP, r);
+                Prof p(g, s, MST_K_COMPOSE, r);
                 MapChain full = chain;
                 full.m[full.len++] = Mr;
                 CK(launch_chain_compose(s, g->nsm, (u32)n, full, g->phi));
                 phi_ready = true;
             }
             cur = g->arcs0;
+            cur_light = false;
             brnd = 0;
             nb_sz = (u32)n;
-            g->hcnt[arec(0, r)] = g->shards[0].A;
-            CK(cudaMemcpyAsync(g->dcnt + arec(0, r), g->hcnt + arec(0, r), sizeof(u32),
-                               cudaMemcpyHostToDevice, s));
+            for (int j = 0; j < G; ++j) {  // every shard re-reads all its records
+                g->hcnt[arec(j, r)] = (u32)(g->shards[j].hi - g->shards[j].lo);
+                CK(cudaMemcpyAsync(g->dcnt + arec(j, r), g->hcnt + arec(j, r), sizeof(u32),
+                                   cudaMemcpyHostToDevice, s));
+            }
         }
         if (moff + nr + nn > 3 * n + 1) return fail(MST_EINTERNAL, "label-map storage overflow");
         bool to_dense = false;
         if (dense) {
             // A9/NEXT-1 dense round: scan the matrix, collapse into the next (smaller) one
-            Prof p(g, s, MST_K_DENSE, r);
+            Prof p(g, s, MST_K_DENSE, r, MST_SUB_DENSE_ROUND);
             CK(launch_dense_init(s, g->nsm, nn, g->mat[mc ^ 1]));
             CK(launch_dense_round(s, g->nsm, nr, g->mat[mc], Mr, nn, g->mat[mc ^ 1], bnxt));
         } else {
@@ -780,7 +1023,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                 Mpass = g->phi;
                 phi_ready = false;
             } else if (brnd < r) {
-                Prof p(g, s, MST_K_JUMP, r);
+                Prof p(g, s, MST_K_COMPOSE, r);
                 const int* src = (brnd == r - 1) ? chain.m[chain.len - 1] : g->phi;
                 CK(launch_compose(s, g->nsm, nb_sz, src, Mr, g->phi));
                 Mpass = g->phi;
@@ -805,9 +1048,9 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             if (adaptive) {
                 cc.tau = g->tau;
                 if (r == 0) {  // no previous pass: sample this pass's records
-                    Prof p(g, s, MST_K_JUMP, r);
+                    Prof p(g, s, MST_K_COMPOSE, r, 1);
                     const Shard& sh = g->shards[dsh];
-                    CK(launch_sample_survival(s, cur + sh.lo, g->dcnt + arec(dsh, r), Mpass,
+                    CK(launch_sample_survival(s, cur + off(sh), g->dcnt + arec(dsh, r), Mpass,
                                               g->dcnt + C_SAMP, g->dcnt + C_SAMP + 1));
                     cc.num = g->dcnt + C_SAMP;
                     cc.den = g->dcnt + C_SAMP + 1;
@@ -819,14 +1062,19 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             for (int j = 0; j < G; ++j) {
                 Shard& sh = g->shards[j];
                 u64* tgt = g->sim ? g->shard_best + (u64)j * n : bnxt;
-                Prof p(g, s, MST_K_FILTER, r);
+                Prof p(g, s, MST_K_FILTER, r,
+                       to_dense ? MST_SUB_TRANSITION
+                       : cur_light ? MST_SUB_LIGHT
+                       : (r == g->st.light_switch_round ? MST_SUB_SWITCH : MST_SUB_SPARSE), j);
                 uint4* out = (never || to_dense) ? nullptr : const_cast<uint4*>(outbuf) + sh.lo;
                 CompactCtl ccj = cc;
                 if (adaptive && j == dsh) {
                     ccj.hword = g->dmap + HSURV + r;
                     ccj.tag = tag_base | (u32)r;
                 }
-                CK(launch_filter_min(s, g->nsm, g->dcnt + arec(j, r), sh.hi - sh.lo, cur + sh.lo,
+                // (a light window holds <= the shard's records + its filler)
+                const u64 amax = (sh.hi - sh.lo) + (cur_light ? (u64)pass_warps(g->nsm) * LBLK_MAX : 0);
+                CK(launch_filter_min(s, g->nsm, g->dcnt + arec(j, r), amax, cur + off(sh),
                                      Mpass, out, tgt, nn, g->status, g->epoch++,
                                      g->dcnt + arec(j, r + 1), g->dcnt + C_TILE, g->pass_seq,
                                      to_dense ? g->mat[0] : nullptr, ccj,
@@ -840,6 +1088,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                 pend_out = outbuf;
             } else if (!never && !to_dense) {
                 cur = outbuf;
+                cur_light = false;
                 brnd = r + 1;
                 nb_sz = nn;
                 g->st.compacted_mask |= 1ll << r;
@@ -851,19 +1100,18 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         if (to_dense) {
             // the transition pass filled only the matrix: every rank needs all of it for the
             // replicated dense rounds, and the first dense round's minima come from it
-            if (g->comm) {
+            if (dist) {
                 Prof p(g, s, MST_K_COMM, r);
-                CKN(ncclAllReduce(g->mat[0], g->mat[0], dense_entries(nn), ncclUint64, ncclMin,
-                                  g->comm, s));
+                CKS(xchg_min(g, s, g->mat[0], dense_entries(nn), false));
             }
-            Prof p(g, s, MST_K_DENSE, r);
+            Prof p(g, s, MST_K_DENSE, r, MST_SUB_DENSE_BEST);
             CK(launch_dense_best(s, g->nsm, nn, g->mat[0], bnxt));
         } else if (g->sim && !dense) {
             Prof p(g, s, MST_K_COMM, r);
             CK(launch_combine_min(s, g->nsm, nn, G, g->shard_best, n, bnxt));
-        } else if (g->comm && !dense) {
+        } else if (dist && !dense) {
             Prof p(g, s, MST_K_COMM, r);
-            CKN(ncclAllReduce(bnxt, bnxt, nn, ncclUint64, ncclMin, g->comm, s));
+            CKS(xchg_min(g, s, bnxt, nn, false));
         }
         if (to_dense) {
             dense = true;
@@ -929,17 +1177,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     *out_total = g->hacc[0];
     g->st.num_edges = *out_num;
     g->st.total_weight = *out_total;
-    if (g->prof) {
-        for (auto& rc : g->recs) {
-            float ms = 0;
-            cudaEventElapsedTime(&ms, rc.a, rc.b);
-            g->st.kernel_ms[rc.kind] += ms;
-            g->st.kernel_launches[rc.kind] += 1;
-            if ((rc.kind == MST_K_FILTER || rc.kind == MST_K_DENSE) && rc.round < MST_MAX_ROUNDS)
-                g->st.round_filter_ms[rc.round] += ms;
-        }
-    }
-    g->st.profiling = g->prof ? 1 : 0;
+    collect_profile(g);
     g->st.gpu_launches = (int64_t)(kernel_launches() - kl0);
     return MST_OK;
 }
@@ -991,6 +1229,15 @@ mst_status mst_create_dist(int64_t n, int64_t m, const int32_t* src, const int32
     return guarded([&]() -> mst_status {
         if (nranks > 1 && !id) return fail(MST_EINVAL, "id is NULL");
         return create_common(n, m, src, dst, w, 1, id, rank, nranks, out);
+    });
+}
+
+mst_status mst_create_dist_hostx(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
+                                 const uint32_t* w, int rank, int nranks,
+                                 mst_allreduce_min_fn fn, void* ctx, mst_graph** out) {
+    return guarded([&]() -> mst_status {
+        if (!fn) return fail(MST_EINVAL, "exchange callback is NULL");
+        return create_common(n, m, src, dst, w, 1, nullptr, rank, nranks, out, true, fn, ctx);
     });
 }
 
@@ -1137,11 +1384,22 @@ mst_status mst_set_option(mst_graph* g, int option, int64_t value) {
             g->opt_tail = value != 0;
         } else if (option == MST_OPT_KEEP_EDGES) {
             g->opt_keep = value != 0;
+        } else if (option == MST_OPT_UNION_FIND) {
+            g->opt_uf = value != 0;
         } else {
             return fail(MST_EINVAL, "unknown option %d", option);
         }
         return MST_OK;
     });
+}
+
+mst_status mst_get_launch_times(const mst_graph* g, mst_launch_time* out, int64_t cap,
+                                int64_t* count) {
+    if (!g || !count || cap < 0 || (cap > 0 && !out)) return fail(MST_EINVAL, "bad argument");
+    const int64_t k = (int64_t)g->ltimes.size();
+    *count = k;
+    for (int64_t i = 0; i < std::min(k, cap); ++i) out[i] = g->ltimes[i];
+    return MST_OK;
 }
 
 mst_status mst_set_profiling(mst_graph* g, int enable) {

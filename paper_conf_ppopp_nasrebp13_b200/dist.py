@@ -31,6 +31,20 @@ def share_unique_id(make_id, group=None) -> bytes:
     return broadcast_bytes(payload, 128, 0, group)
 
 
+def allreduce_min_u64_(words, group=None) -> None:
+    """In place: words (numpy uint64) <- their element-wise minimum over all ranks. The
+    exchange of mst_create_dist_hostx (test aid) over any backend: uint64 -> int64 by flipping
+    the sign bit preserves the order, so the backend's signed MIN is the unsigned MIN."""
+    import numpy as np
+    flip = np.uint64(1 << 63)
+    t = torch.from_numpy((words ^ flip).view(np.int64).copy())
+    dev = _device_for(group)
+    if dev.type != "cpu":
+        t = t.to(dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
+    words[:] = t.cpu().numpy().view(np.uint64) ^ flip
+
+
 def max_over_ranks(x: float, group=None) -> float:
     """The bench's timing rule: the slowest rank's time."""
     t = torch.tensor([float(x)], dtype=torch.float64, device=_device_for(group))

@@ -18,17 +18,26 @@ MST_OK, MST_EINVAL, MST_ENOMEM, MST_ECUDA, MST_ENCCL, MST_EINTERNAL, MST_ENOTSUP
 STATUS_NAMES = {0: "MST_OK", 1: "MST_EINVAL", 2: "MST_ENOMEM", 3: "MST_ECUDA", 4: "MST_ENCCL",
                 5: "MST_EINTERNAL", 6: "MST_ENOTSUP"}
 MAX_ROUNDS = 64
-K_INIT, K_MIN0, K_HOOK, K_JUMP, K_FILTER, K_OUTPUT, K_COMM, K_DENSE, K_COUNT = range(9)
-KERNEL_NAMES = ["init", "min0", "hook", "jump", "filter", "output", "comm", "dense"]
+K_INIT, K_MIN0, K_HOOK, K_JUMP, K_FILTER, K_OUTPUT, K_COMM, K_DENSE, K_LIGHT, K_COMPOSE, \
+    K_COUNT = range(11)
+KERNEL_NAMES = ["init", "min0", "hook", "jump", "filter", "output", "comm", "dense", "light",
+                "compose"]
+# launch sub-kinds per kind (include/mst.h MST_SUB_*)
+SUB_NAMES = {K_MIN0: ["min_all", "extract", "min_light"],
+             K_FILTER: ["sparse", "light", "switch", "transition"],
+             K_DENSE: ["dense_round", "dense_best", "tail"],
+             K_COMPOSE: ["compose", "sample"]}
 
 # every symbol include/mst.h declares
-DEBUG_EXPORTS = ["mst_debug_filter_pass", "mst_shard_ranges"]  # include/mst_debug.h
+DEBUG_EXPORTS = ["mst_debug_filter_pass", "mst_shard_ranges",
+                 "mst_create_dist_hostx"]  # include/mst_debug.h
 EXPORTS = ["mst_create", "mst_create_host", "mst_run", "mst_run_host", "mst_solve_host",
            "mst_destroy", "mst_last_error", "mst_get_stats", "mst_set_profiling",
            "mst_get_unique_id", "mst_create_dist", "mst_create_sim", "mst_version",
-           "mst_set_option"]
+           "mst_set_option", "mst_get_launch_times"]
 MST_OPT_DENSE, MST_OPT_KEEP_EDGES, MST_OPT_DEVICE_TAIL, MST_OPT_COMPACT_TAU = 1, 2, 3, 4
 MST_OPT_LIGHT_FIRST = 5
+MST_OPT_UNION_FIND = 6
 
 
 class mst_stats(ctypes.Structure):
@@ -49,6 +58,16 @@ class mst_stats(ctypes.Structure):
         ("light_switch_round", ctypes.c_int32),
         ("light_t", ctypes.c_uint32),
     ]
+
+
+# include/mst_debug.h: int (*)(uint64_t* host_buf, int64_t count, void* ctx)
+ALLREDUCE_MIN_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.POINTER(ctypes.c_uint64), ctypes.c_int64,
+                                    ctypes.c_void_p)
+
+
+class mst_launch_time(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int32), ("sub", ctypes.c_int32), ("round", ctypes.c_int32),
+                ("shard", ctypes.c_int32), ("ms", ctypes.c_double)]
 
 
 class MSTError(RuntimeError):
@@ -88,6 +107,8 @@ def load(build_if_missing: bool = True):
     L.mst_last_error.restype = ctypes.c_char_p
     L.mst_get_stats.argtypes = [p, ctypes.POINTER(mst_stats)]
     L.mst_set_profiling.argtypes = [p, i32]
+    L.mst_get_launch_times.argtypes = [p, ctypes.POINTER(mst_launch_time), i64,
+                                       ctypes.POINTER(ctypes.c_int64)]
     L.mst_set_option.argtypes = [p, i32, i64]
     L.mst_get_unique_id.argtypes = [p]
     L.mst_version.restype = ctypes.c_char_p
@@ -96,6 +117,8 @@ def load(build_if_missing: bool = True):
     L.mst_debug_filter_pass.restype = ctypes.c_int
     L.mst_shard_ranges.argtypes = [p, i64, i32, p, p]
     L.mst_shard_ranges.restype = ctypes.c_int
+    L.mst_create_dist_hostx.argtypes = [i64, i64, p, p, p, i32, i32, ALLREDUCE_MIN_FN, p, pp]
+    L.mst_create_dist_hostx.restype = ctypes.c_int
     for name in EXPORTS:
         if name not in ("mst_destroy", "mst_last_error", "mst_version"):
             getattr(L, name).restype = ctypes.c_int
@@ -132,10 +155,12 @@ def mst_get_unique_id() -> bytes:
 
 class MSTGraph:
     """Owns one library handle. Construct with device tensors (mst_create), host arrays
-    (``host=True``: mst_create_host), ``nshards`` (mst_create_sim) or ``dist=(id, rank,
-    nranks)`` (mst_create_dist)."""
+    (``host=True``: mst_create_host), ``nshards`` (mst_create_sim), ``dist=(id, rank,
+    nranks)`` (mst_create_dist) or ``hostx=(rank, nranks, fn)`` (mst_create_dist_hostx: the
+    exchange is ``fn(words)``, which must replace the numpy uint64 array ``words`` in place by
+    its element-wise minimum over all ranks)."""
 
-    def __init__(self, n, src, dst, w, *, host=False, nshards=1, dist=None):
+    def __init__(self, n, src, dst, w, *, host=False, nshards=1, dist=None, hostx=None):
         L = load()
         self.n = int(n)
         self.m = int(src.shape[0])
@@ -154,7 +179,22 @@ class MSTGraph:
                     raise ValueError("src/dst/w must be contiguous CUDA tensors")
                 if t.dtype not in (dt, torch.uint32) or t.element_size() != 4:
                     raise ValueError("src/dst must be int32 and w 32-bit")
-            if dist is not None:
+            if hostx is not None:
+                rank, nranks, fn = hostx
+
+                def _cb(buf, count, _ctx, fn=fn):
+                    try:
+                        fn(np.ctypeslib.as_array(buf, shape=(int(count),)))
+                        return 0
+                    except Exception:  # noqa: BLE001 -> MST_ENCCL from mst_run
+                        import traceback
+                        traceback.print_exc()
+                        return 1
+                self._xcb = ALLREDUCE_MIN_FN(_cb)  # kept alive with the handle
+                _check(L.mst_create_dist_hostx(self.n, self.m, _dptr(src), _dptr(dst), _dptr(w),
+                                               int(rank), int(nranks), self._xcb, None,
+                                               ctypes.byref(h)))
+            elif dist is not None:
                 uid, rank, nranks = dist
                 idbuf = (ctypes.c_uint8 * 128).from_buffer_copy(uid)
                 _check(L.mst_create_dist(self.n, self.m, _dptr(src), _dptr(dst), _dptr(w),
@@ -215,6 +255,21 @@ class MSTGraph:
             "light_switch_round": s.light_switch_round,
             "light_t": s.light_t,
         }
+
+    def launch_times(self) -> list:
+        """Per-launch event times of the last profiled run: dicts {kind, sub, round, shard, ms}
+        (kind/sub as names, include/mst.h MST_K_* / MST_SUB_*)."""
+        cnt = ctypes.c_int64(0)
+        _check(load().mst_get_launch_times(self._h, None, 0, ctypes.byref(cnt)))
+        buf = (mst_launch_time * max(cnt.value, 1))()
+        _check(load().mst_get_launch_times(self._h, buf, cnt.value, ctypes.byref(cnt)))
+        out = []
+        for x in buf[: cnt.value]:
+            subs = SUB_NAMES.get(x.kind)
+            out.append({"kind": KERNEL_NAMES[x.kind],
+                        "sub": subs[x.sub] if subs and x.sub < len(subs) else str(x.sub),
+                        "round": x.round, "shard": x.shard, "ms": x.ms})
+        return out
 
     def debug_filter_pass(self, map_kind=0, group=1, iters=5, stream=None):
         """Times the A8 kernel alone on the round-0 arcs (include/mst_debug.h)."""

@@ -33,7 +33,13 @@ def dev(a):
     return torch.from_numpy(a.astype(np.int32, copy=False)).to("cuda")
 
 
+# MST_TEST_OPTIONS="6=1,4=0": run options applied to every case (option=value, include/mst.h)
+EXTRA = [tuple(int(x) for x in kv.split("=")) for kv in
+         os.environ.get("MST_TEST_OPTIONS", "").split(",") if kv]
+
+
 def check(name, n, src, dst, w, options=()):
+    options = list(options) + EXTRA
     src = np.asarray(src, np.int32)
     dst = np.asarray(dst, np.int32)
     w32 = np.asarray(w, np.uint64).astype(np.uint32)

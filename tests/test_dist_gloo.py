@@ -53,8 +53,14 @@ def _worker(rank, port, results):
         mine = (int(lo[rank]), int(hi[rank]))
         wins = [None] * WORLD
         dist.all_gather_object(wins, mine)
+        # 4. the host exchange's unsigned MIN (mst_create_dist_hostx): values above 2^63 and
+        #    the "no edge" key 2^64 - 1 must order as unsigned
+        words = np.array([5, 2**64 - 1, 2**63 + 7, 2**63 - 1, 0], np.uint64)
+        if rank == 1:
+            words = np.array([9, 2**63 + 3, 2**63 + 9, 2**64 - 2, 1], np.uint64)
+        mdist.allreduce_min_u64_(words)
         results[rank] = {"ids": ids, "t": t, "wins": wins, "row_end": int(row[-1]),
-                         "lo": lo.tolist(), "hi": hi.tolist()}
+                         "lo": lo.tolist(), "hi": hi.tolist(), "words": words.tolist()}
     finally:
         dist.destroy_process_group()
 
@@ -69,6 +75,7 @@ def test_gloo_world2_host_logic():
     r0, r1 = results[0], results[1]
     assert r0["ids"][0] == r0["ids"][1] == r1["ids"][0] and len(r0["ids"][0]) == 128
     assert r0["t"] == r1["t"] == 11.0
+    assert r0["words"] == r1["words"] == [5, 2**63 + 3, 2**63 + 7, 2**63 - 1, 0]
     # identical partitions on both ranks; contiguous, disjoint, covering [0, arcs)
     assert r0["wins"] == r1["wins"]
     wins = r0["wins"]

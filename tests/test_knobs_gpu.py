@@ -38,6 +38,9 @@ KNOBS = [
     {"MST_LIGHT_K": "1"},
     {"MST_LIGHT_ONLY0": "1"},
     {"MST_LIGHT_ONLY0": "0"},
+    {"MST_TEST_OPTIONS": "6=1"},                     # union-find variant (NEXT-3)
+    {"MST_TEST_OPTIONS": "6=1", "MST_UF_TAG": "0"},  # ... untagged keys, best reset per round
+    {"MST_TEST_OPTIONS": "6=1,4=1000"},              # ... always compacting
 ]
 
 

@@ -495,3 +495,65 @@ def test_output_dense_forest_tiles(lib, oracle_mod):
     dst = np.concatenate([ps + 1, ed]).astype(np.int32)
     w = np.concatenate([rng.integers(0, 10, n - 1), rng.integers(10, 1000, extra)]).astype(np.uint32)
     assert_parity(lib, oracle_mod, n, src, dst, w, runs=2)
+
+
+# ------------------------------------------------------------------ NEXT-3: union-find variant
+UF = 6  # MST_OPT_UNION_FIND (include/mst.h)
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_union_find_random_multigraphs(lib, oracle_mod, seed):
+    rng = np.random.default_rng(5000 + seed)
+    n = int(rng.integers(1, 20_000))
+    m = int(rng.integers(0, 8 * n))
+    wmax = [0, 1, 7, 1000, 2**32 - 1][seed % 5]
+    src, dst, w = mc.random_multigraph(rng, n, m, wmax)
+    st = assert_parity(lib, oracle_mod, n, src, dst, w, runs=2, options=[(UF, 1)])
+    assert st["dense_round"] == -1 and st["light_t"] == 0xFFFFFFFF
+
+
+@pytest.mark.parametrize("tau", [0, 500, 900, 1000])
+@pytest.mark.parametrize("k,sd", [(1, 0), (2, 6), (3, 8), (4, 6), (5, 6)])
+def test_union_find_configs(lib, oracle_mod, gg, k, sd, tau):
+    g = gg.config(k, s=9, scale_down=sd)
+    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, runs=2,
+                       options=[(UF, 1), (lib.mst.MST_OPT_COMPACT_TAU, tau)])
+    assert not st["compacted"][0]  # round 0: every non-loop record crosses two singletons
+    if tau == 0:
+        assert all(a == st["arcs0"] for a in st["a_r"])  # the records are never touched
+    assert st["n_r"][0] == g.n and all(a >= b for a, b in zip(st["n_r"], st["n_r"][1:]))
+
+
+@pytest.mark.parametrize("k", [1, 2, 3, 4, 5])
+def test_union_find_full_size(lib, oracle_mod, gg, k):
+    g = gg.config(k)
+    assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, options=[(UF, 1)])
+
+
+def test_union_find_adversarial(lib, oracle_mod):
+    # monotone path: every union links the next vertex, one chain of depth n - 1
+    n = 300_000
+    src = np.arange(n - 1, dtype=np.int32)
+    assert_parity(lib, oracle_mod, n, src, src + 1, np.arange(1, n, dtype=np.uint32),
+                  options=[(UF, 1)])
+    assert_parity(lib, oracle_mod, n, src, src + 1, np.arange(n - 1, 0, -1).astype(np.uint32),
+                  options=[(UF, 1)])
+    # star of degree 10^6 with extra cross edges; empty and degenerate inputs
+    n = 1_000_001
+    rng = np.random.default_rng(4)
+    src = np.zeros(n - 1, np.int32)
+    dst = np.arange(1, n, dtype=np.int32)
+    w = rng.integers(0, 1000, n - 1).astype(np.uint32)
+    assert_parity(lib, oracle_mod, n, src, dst, w, options=[(UF, 1)])
+    for n, s_, d_, w_ in [(0, [], [], []), (1, [], [], []), (5, [], [], []),
+                          (3, [0, 1, 2], [0, 1, 2], [1, 2, 3]), (2, [1, 0, 1], [0, 1, 0], [3, 3, 3])]:
+        assert_parity(lib, oracle_mod, n, s_, d_, w_, options=[(UF, 1)])
+
+
+def test_union_find_single_gpu_only(lib, gg):
+    g = gg.config(1)
+    with lib.MSTGraph(g.n, dev(g.src), dev(g.dst), dev(g.w), nshards=2) as h:
+        h.set_option(UF, 1)
+        with pytest.raises(lib.MSTError) as e:
+            h.run()
+        assert e.value.status == 6  # MST_ENOTSUP
