@@ -268,10 +268,15 @@ def run_gpu(args):
             round_acc = [{"r": r, "kind": bm[r]["kind"], "n_r": st["n_r"][r], "A_r": st["a_r"][r],
                           "compacted": bm[r].get("compacted"),
                           "survival_permille": st["survival_permille"][r],
-                          "filter_ms": 0.0, "filter_bytes": bm[r]["bytes"]}
+                          "filter_ms": 0.0, "filter_bytes": bm[r]["bytes"],
+                          "hook_ms": 0.0, "jump_ms": 0.0, "compose_ms": 0.0}
                          for r in range(st["rounds"])]
         for r in range(st["rounds"]):
             round_acc[r]["filter_ms"] += st["round_filter_ms"][r] / args.steps
+        for lt in h.launch_times():  # per-round hook / jump / compose times
+            key = lt["kind"] + "_ms"
+            if 0 <= lt["round"] < len(round_acc) and key in round_acc[lt["round"]]:
+                round_acc[lt["round"]][key] += lt["ms"] / args.steps
     h.set_profiling(False)
     barrier()
     clk = clocks.stop()
