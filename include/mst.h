@@ -129,7 +129,8 @@ enum {
     MST_K_DENSE = 7,   /* A9 dense rounds over the component min-matrix              */
     MST_K_LIGHT = 8,   /* A2 light-edge threshold select (sampled radix select)       */
     MST_K_COMPOSE = 9, /* A7 label-map composition (+ the round-0 survival sample)    */
-    MST_K_COUNT = 10
+    MST_K_SMALL = 10,  /* A1-A11 in one CTA (MST_OPT_SMALL: graphs that fit smem)      */
+    MST_K_COUNT = 11
 };
 /* launch sub-kinds (mst_launch_time.sub), so unlike launches of one kind are told apart:
  *   MST_K_MIN0  : MIN_ALL   = minima over every record (+ the light-record write);
@@ -234,12 +235,19 @@ mst_status mst_set_profiling(mst_graph* g, int enable);
  *       min-reduces per root, and unions the two roots of every chosen edge by CAS. No
  *       renumbering, no label maps, no dense rounds, no light-edge phase. Single-GPU handles
  *       only (MST_ENOTSUP from mst_run otherwise). Never changes the result.
+ *   MST_OPT_SMALL (default 1): graphs whose edge records (16 B each), per-vertex arrays
+ *       (16 B per vertex) and forest bits fit one CTA's shared memory (~220 KB; grid64: 197 KB)
+ *       run every round in ONE launch on one SM (kernels.cu k_small_msf: minima with the
+ *       partner in packed keys, hook, path-halving jumps, block-scan renumbering, relabel and
+ *       deletion, ascending ids): the latency regime of row A10, where the multi-kernel path
+ *       pays launches and a host wait per round for microseconds of work. Single-GPU handles
+ *       without MST_OPT_KEEP_EDGES / MST_OPT_UNION_FIND; 0 = always the multi-kernel path.
  * Keys of the component minima (rows A2/A8): (uint64(w) << 32) | eid, or, when the largest
  * weight, the largest edge id and the largest vertex id fit 63 bits together, the packed
  * (w << s1) | (eid << pb) | partner label — the same (w, eid) order (reading R17).
  */
 enum { MST_OPT_DENSE = 1, MST_OPT_KEEP_EDGES = 2, MST_OPT_DEVICE_TAIL = 3, MST_OPT_COMPACT_TAU = 4,
-       MST_OPT_LIGHT_FIRST = 5, MST_OPT_UNION_FIND = 6 };
+       MST_OPT_LIGHT_FIRST = 5, MST_OPT_UNION_FIND = 6, MST_OPT_SMALL = 7 };
 mst_status mst_set_option(mst_graph* g, int option, int64_t value);
 
 /* ------------------------------------------------------------------ multi-GPU (§8(e))

@@ -116,6 +116,15 @@ cudaError_t launch_dense_tail(cudaStream_t st, int nsm, u32 n0, u64* best0, u64*
 cudaError_t launch_compose(cudaStream_t st, int nsm, u32 nb, const int* src, const int* Mr, int* phi);
 cudaError_t launch_sample_survival(cudaStream_t st, const uint4* in, const u32* a_ptr, const int* M,
                                    u32* num, u32* den);
+// A10 latency regime: the whole method in one CTA (records, component arrays and forest bits
+// in shared memory) when small_smem_bytes(n, E, nwords) <= small_smem_limit() and packed keys
+// (w << s1 | eid << pb | partner) fit 64 bits; res (device, small_out_bytes()) receives
+// {count, rounds, total, n_r[64], a_r[64]}
+size_t small_smem_bytes(u64 n, u64 E, u64 nwords);
+size_t small_smem_limit();
+size_t small_out_bytes();
+cudaError_t launch_small(cudaStream_t st, u32 n, u32 E, u32 nwords, const uint4* arcs, u32 s1,
+                         u32 pb, int* out, void* res);
 // max_ids: an upper bound of the forest size (n - 1) — sizes the staging of the id writes
 cudaError_t launch_output(cudaStream_t st, u32 nwords, const u32* msf, int* out, u32* tcnt,
                           u32* out_count, u32 max_ids);

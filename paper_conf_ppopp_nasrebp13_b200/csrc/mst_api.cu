@@ -152,6 +152,9 @@ struct mst_graph {
     u64 A0_local = 0;                    // records built on this rank (all shards)
 
     bool opt_uf = false;     // MST_OPT_UNION_FIND (NEXT-3 variant)
+    bool opt_small = true;   // MST_OPT_SMALL (one-CTA path for graphs that fit shared memory)
+    void* small_res = nullptr;   // its device result block (SmallOut)
+    void* small_host = nullptr;  // pinned copy
     bool opt_dense = true;   // MST_OPT_DENSE
     bool opt_keep = false;   // MST_OPT_KEEP_EDGES (paper-faithful ablation)
     bool opt_tail = true;    // MST_OPT_DEVICE_TAIL
@@ -212,6 +215,7 @@ void release(mst_graph* g) {
     if (g->hacc) cudaFreeHost(g->hacc);
     if (g->hmap) cudaFreeHost((void*)g->hmap);
     if (g->xhost) cudaFreeHost(g->xhost);
+    if (g->small_host) cudaFreeHost(g->small_host);
     if (g->trace) cudaFree(g->trace);
     for (auto e : g->evpool) cudaEventDestroy(e);
     if (g->fail_ev) cudaEventDestroy(g->fail_ev);
@@ -410,6 +414,8 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     // defers components (no merge) and switches to all edges before 3n + 1 is reached
     CKS(galloc(g, &g->maps, 3 * n + 1));
     CKS(galloc(g, &g->msf, g->nwords));
+    CKS(galloc(g, reinterpret_cast<unsigned char**>(&g->small_res), small_out_bytes()));
+    CK(cudaMallocHost(&g->small_host, small_out_bytes()));
     CKS(galloc(g, &g->phi, n));
     if (n >= 2) {  // dense min-matrices (A9 / NEXT-1), <= 67 MB each
         CKS(galloc(g, &g->mat[0], dense_entries(n)));
@@ -584,6 +590,60 @@ void collect_profile(mst_graph* g) {
     g->st.profiling = g->prof ? 1 : 0;
 }
 
+// ---------------------------------------------------------------- A10: the one-CTA path
+// Graphs whose records, per-component arrays and forest bits fit one CTA's shared memory run
+// the whole method in one launch (kernels.cu k_small_msf): no per-round launches, no host
+// round trips (grid64: ~10 launches and a host wait per round for microseconds of work).
+u32 bits_of(u64 x) { u32 b = 0; while (x) { ++b; x >>= 1; } return b; }
+bool small_ok(const mst_graph* g) {
+    static const char* e = getenv("MST_SMALL");  // "0": never (ablation)
+    if (!g->opt_small || (e && e[0] == '0') || g->opt_keep || g->shards.size() != 1 ||
+        g->xkind != X_NONE || g->n < 2)
+        return false;
+    const u64 E = g->shards[0].hi - g->shards[0].lo;
+    const u32 pb = bits_of((u64)g->n - 1), eb = bits_of(g->m > 0 ? (u64)g->m - 1 : 0);
+    return bits_of(g->hcnt[C_WMAX]) + eb + pb <= 64 &&
+           small_smem_bytes((u64)g->n, E, g->nwords) <= small_smem_limit();
+}
+struct SmallHost {  // (the layout of kernels.cu SmallOut)
+    u32 count, rounds;
+    u64 total;
+    u32 n_r[64], a_r[64];
+};
+mst_status run_small(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out_num,
+                     uint64_t* out_total, unsigned long long kl0) {
+    static_assert(sizeof(SmallHost) == 8 + 8 + 512, "SmallOut layout");
+    const u64 n = g->n, E = g->shards[0].hi - g->shards[0].lo;
+    const u32 pb = bits_of(n - 1), eb = bits_of(g->m > 0 ? (u64)g->m - 1 : 0);
+    {
+        Prof p(g, s, MST_K_SMALL, 0);
+        CK(launch_small(s, (u32)n, (u32)E, (u32)g->nwords, g->arcs0 + g->shards[0].lo, eb + pb, pb,
+                        out_ids, g->small_res));
+    }
+    CK(cudaMemcpyAsync(g->small_host, g->small_res, sizeof(SmallHost), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    const SmallHost* h = reinterpret_cast<const SmallHost*>(g->small_host);
+    g->st.rounds = (int32_t)std::min<u32>(h->rounds, MST_MAX_ROUNDS);
+    for (int r = 0; r < g->st.rounds; ++r) {
+        g->st.n_r[r] = h->n_r[r];
+        g->st.a_r[r] = h->a_r[r];
+    }
+    g->st.dense_round = -1;
+    g->st.light_switch_round = -1;
+    g->st.light_t = 0xffffffffu;
+    g->st.compacted_mask = 0;
+    g->st.hub_row = 0;
+    for (int i = 0; i < MST_MAX_ROUNDS; ++i) g->st.survival_permille[i] = -1;
+    if ((u64)h->count >= n) return fail(MST_EINTERNAL, "forest has >= n edges");
+    *out_num = (int64_t)h->count;
+    *out_total = h->total;
+    g->st.num_edges = *out_num;
+    g->st.total_weight = *out_total;
+    collect_profile(g);
+    g->st.gpu_launches = (int64_t)(kernel_launches() - kl0);
+    return MST_OK;
+}
+
 // ---------------------------------------------------------------- NEXT-3: union-find variant
 // Bulk-synchronous Boruvka over the unmodified edge records with a union-find (§8.4
 // L389; kernels in kernels.cu "NEXT-3"). Per round r: K1 = k_arc_pass<MODE_UF>
@@ -735,6 +795,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         return MST_OK;
     }
     if (g->opt_uf) return run_uf(g, s, out_ids, out_num, out_total, kl0);
+    if (small_ok(g)) return run_small(g, s, out_ids, out_num, out_total, kl0);
     const int G = (int)g->shards.size();
     // ---- A1 init
     {
@@ -1386,6 +1447,8 @@ mst_status mst_set_option(mst_graph* g, int option, int64_t value) {
             g->opt_keep = value != 0;
         } else if (option == MST_OPT_UNION_FIND) {
             g->opt_uf = value != 0;
+        } else if (option == MST_OPT_SMALL) {
+            g->opt_small = value != 0;
         } else {
             return fail(MST_EINVAL, "unknown option %d", option);
         }

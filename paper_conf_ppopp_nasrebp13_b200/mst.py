@@ -19,9 +19,9 @@ STATUS_NAMES = {0: "MST_OK", 1: "MST_EINVAL", 2: "MST_ENOMEM", 3: "MST_ECUDA", 4
                 5: "MST_EINTERNAL", 6: "MST_ENOTSUP"}
 MAX_ROUNDS = 64
 K_INIT, K_MIN0, K_HOOK, K_JUMP, K_FILTER, K_OUTPUT, K_COMM, K_DENSE, K_LIGHT, K_COMPOSE, \
-    K_COUNT = range(11)
+    K_SMALL, K_COUNT = range(12)
 KERNEL_NAMES = ["init", "min0", "hook", "jump", "filter", "output", "comm", "dense", "light",
-                "compose"]
+                "compose", "small"]
 # launch sub-kinds per kind (include/mst.h MST_SUB_*)
 SUB_NAMES = {K_MIN0: ["min_all", "extract", "min_light"],
              K_FILTER: ["sparse", "light", "switch", "transition"],
@@ -38,6 +38,7 @@ EXPORTS = ["mst_create", "mst_create_host", "mst_run", "mst_run_host", "mst_solv
 MST_OPT_DENSE, MST_OPT_KEEP_EDGES, MST_OPT_DEVICE_TAIL, MST_OPT_COMPACT_TAU = 1, 2, 3, 4
 MST_OPT_LIGHT_FIRST = 5
 MST_OPT_UNION_FIND = 6
+MST_OPT_SMALL = 7
 
 
 class mst_stats(ctypes.Structure):

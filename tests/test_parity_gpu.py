@@ -29,11 +29,18 @@ def dev(a, dt=torch.int32):
     return torch.from_numpy(a.astype(np.int32, copy=False)).to("cuda")
 
 
-def gpu_msf(lib, n, src, dst, w, nshards=1, runs=1, options=()):
+SMALL = 7  # MST_OPT_SMALL (include/mst.h)
+
+
+def gpu_msf(lib, n, src, dst, w, nshards=1, runs=1, options=(), small=False):
+    """small=False (the default here) keeps every test on the multi-kernel path even for
+    graphs the one-CTA path (MST_OPT_SMALL) would take; the small-path tests pass True."""
     src = np.asarray(src, np.int32)
     dst = np.asarray(dst, np.int32)
     w = np.asarray(w, np.uint64).astype(np.uint32)
     with lib.MSTGraph(n, dev(src), dev(dst), dev(w), nshards=nshards) as g:
+        if not small:
+            g.set_option(SMALL, 0)
         for opt, val in options:
             g.set_option(opt, val)
         outs = []
@@ -46,8 +53,8 @@ def gpu_msf(lib, n, src, dst, w, nshards=1, runs=1, options=()):
     return outs[0][0], outs[0][1], outs[0][2], st
 
 
-def assert_parity(lib, oracle_mod, n, src, dst, w, nshards=1, runs=1, options=()):
-    ids, cnt, tot, st = gpu_msf(lib, n, src, dst, w, nshards, runs, options)
+def assert_parity(lib, oracle_mod, n, src, dst, w, nshards=1, runs=1, options=(), small=False):
+    ids, cnt, tot, st = gpu_msf(lib, n, src, dst, w, nshards, runs, options, small)
     o_ids, o_tot = oracle_mod.kruskal(n, src, dst, w)
     assert cnt == len(o_ids), (cnt, len(o_ids))
     assert tot == o_tot, (tot, o_tot)
@@ -557,3 +564,48 @@ def test_union_find_single_gpu_only(lib, gg):
         with pytest.raises(lib.MSTError) as e:
             h.run()
         assert e.value.status == 6  # MST_ENOTSUP
+
+
+# ------------------------------------------------------------------ A10: the one-CTA path
+def _small_used(st):
+    return st["kernel_launches"].get("small", 0) > 0 if st["profiling"] else st["gpu_launches"] == 1
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_small_path_random_multigraphs(lib, oracle_mod, seed):
+    """graphs that fit one CTA's shared memory run every round in one launch (the default)"""
+    rng = np.random.default_rng(8000 + seed)
+    n = int(rng.integers(2, 4000))
+    m = int(rng.integers(0, min(9000, 6 * n)))
+    wmax = [0, 1, 7, 1000, 2**32 - 1][seed % 5]
+    src, dst, w = mc.random_multigraph(rng, n, m, wmax)
+    st = assert_parity(lib, oracle_mod, n, src, dst, w, runs=2, small=True)
+    assert st["gpu_launches"] == 1  # the whole method in one kernel
+
+
+@pytest.mark.parametrize("seed", range(20))
+def test_small_path_tiny_vs_brute_force(lib, seed):
+    rng = np.random.default_rng(300 + seed)
+    n = int(rng.integers(1, 7)); m = int(rng.integers(0, 11))
+    src, dst, w = mc.random_multigraph(rng, n, m, 2)
+    ids, cnt, tot, _ = gpu_msf(lib, n, src, dst, w, small=True)
+    bf, bf_w, _ = mc.brute_force_msf(n, src, dst, w)
+    assert list(ids) == bf and tot == bf_w
+
+
+def test_small_path_grid64_and_edges(lib, oracle_mod, gg):
+    g = gg.config(1)  # grid64: the BASELINE config the one-CTA path exists for
+    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, runs=3, small=True)
+    assert st["gpu_launches"] == 1 and st["rounds"] >= 3
+    assert st["n_r"][0] == g.n and st["a_r"][0] == st["arcs0"]
+    for n, s_, d_, w_ in [(1, [], [], []), (5, [], [], []), (3, [0, 1, 2], [0, 1, 2], [1, 2, 3]),
+                          (2, [0], [1], [2**32 - 1]), (2, [1, 0, 1], [0, 1, 0], [3, 3, 3])]:
+        assert_parity(lib, oracle_mod, n, s_, d_, w_, small=True)
+    # a monotone path (every vertex hooks left: one chain of depth n - 1 in one CTA)
+    n = 6000
+    src = np.arange(n - 1, dtype=np.int32)
+    assert_parity(lib, oracle_mod, n, src, src + 1, np.arange(1, n, dtype=np.uint32), small=True)
+    # a graph just too large for shared memory takes the multi-kernel path
+    g = gg.config(2, scale_down=8)  # n = 16 K, m = 64 K
+    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, small=True)
+    assert st["gpu_launches"] > 1
