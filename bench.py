@@ -135,11 +135,14 @@ def byte_model(st):
     to the dense matrix writes no records (they go to the L2-resident matrix). dense round r (A9): 8 B per matrix entry read (n_r (n_r - 1) / 2 entries).
     The last round only hooks (<= 1 live component is left) and moves no arcs."""
     a, R, dr = st["a_r"], st["rounds"], st.get("dense_round", -1)
+    me = st.get("member_ends", [-1] * R)
     out = []
     for r in range(R):
         dense = dr >= 0 and r >= dr
         if r == R - 1:
             out.append({"kind": "hook-only", "bytes": 0})
+        elif me[r] >= 0:  # member-scan round: the record ends it read (16 B each)
+            out.append({"kind": "member", "compacted": False, "bytes": 16 * me[r]})
         elif dense:
             out.append({"kind": "dense", "bytes": 8 * a[r]})
         else:
@@ -275,7 +278,7 @@ def run_gpu(args):
             round_acc[r]["filter_ms"] += st["round_filter_ms"][r] / args.steps
         for lt in h.launch_times():  # per-round hook / jump / compose times
             key = lt["kind"] + "_ms"
-            if 0 <= lt["round"] < len(round_acc) and key in round_acc[lt["round"]]:
+            if lt["kind"] in ("hook", "jump", "compose") and 0 <= lt["round"] < len(round_acc):
                 round_acc[lt["round"]][key] += lt["ms"] / args.steps
     h.set_profiling(False)
     barrier()

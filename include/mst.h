@@ -138,11 +138,14 @@ enum {
  *                 MIN_LIGHT = minima over the light records
  *   MST_K_FILTER: SPARSE = a pass over the alive records; LIGHT = a light-edge phase pass;
  *                 SWITCH = the pass that re-reads every record after the light phase;
- *                 TRANSITION = the pass into the dense min-matrix
+ *                 TRANSITION = the pass into the dense min-matrix; MEMBER = a member-scan round
+ *                 (the minima of the components outside the top hub's from their members'
+ *                 records, after the light-edge phase)
  *   MST_K_DENSE : DENSE_ROUND, DENSE_BEST, TAIL (the cooperative device tail) */
 enum {
     MST_SUB_MIN_ALL = 0, MST_SUB_EXTRACT = 1, MST_SUB_MIN_LIGHT = 2,
     MST_SUB_SPARSE = 0, MST_SUB_LIGHT = 1, MST_SUB_SWITCH = 2, MST_SUB_TRANSITION = 3,
+    MST_SUB_MEMBER = 4,
     MST_SUB_DENSE_ROUND = 0, MST_SUB_DENSE_BEST = 1, MST_SUB_TAIL = 2
 };
 typedef struct {
@@ -173,6 +176,8 @@ typedef struct {
                                              heavy ones), -1 = not reached / phase off    */
     uint32_t light_t;                     /* its weight threshold (light: w <= light_t);
                                              0xffffffff when the phase was off            */
+    int64_t member_ends[MST_MAX_ROUNDS];  /* member-scan round r: record ends read (the
+                                             members' own + reverse records); -1: not one */
 } mst_stats;
 
 mst_status mst_get_stats(const mst_graph* g, mst_stats* out);

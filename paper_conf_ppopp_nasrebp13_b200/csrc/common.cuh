@@ -15,6 +15,9 @@ typedef uint32_t u32;
 typedef uint64_t u64;
 
 constexpr u64 KEY_INF = ~0ull;          // "no edge" (SURVEY.md §8 notation: ∞ = UINT64_MAX)
+// "not looked at this round" (the member-scan rounds defer the component of the top hub): no
+// real key takes this value (packed keys use < 64 bits; (w << 32 | eid) has eid < 2^31)
+constexpr u64 KEY_DEFER = ~1ull;
 constexpr u32 FULL = 0xffffffffu;
 
 // ------------------------------------------------------------------ memory access

@@ -37,7 +37,7 @@ struct CompactCtl {
 };
 
 cudaError_t launch_degree(cudaStream_t st, int nsm, u32 n, u32 m, const int* src, const int* dst,
-                          u32* eu, u32* ev, u32* deg, u32* err);
+                          const unsigned* w, u32* eu, u32* ev, u32* deg, u32* err, u32* wmax);
 cudaError_t launch_scan_rows(cudaStream_t st, u32 n, const u32* deg, u32* row, u32* cursor,
                              u64* status, u32 epoch);
 cudaError_t launch_reorder(cudaStream_t st, int nsm, u32 n, u32 m, const u32* deg, u32* degn,
@@ -48,7 +48,7 @@ cudaError_t launch_owner_degree(cudaStream_t st, int nsm, u32 m, const u32* eu, 
                                 u32* odeg, int hi_owner);
 cudaError_t launch_scatter(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
                            const unsigned* w, u32* cursor, uint4* arcs, uint2* euv,
-                           int hi_owner, u32* wmax, u32 vlo, u32 vhi, u32 wbase);
+                           int hi_owner, u32 kfmt, u32 vlo, u32 vhi, u32 wbase);
 // (only the records of owners in [vlo, vhi), at their CSR position minus wbase)
 // light_out != nullptr (MST_OPT_LIGHT_FIRST): also append the records of weight <= *light_t
 // to light_out; every consumer warp reserves blocks of light_blk records (one atomic each)
@@ -72,7 +72,8 @@ cudaError_t launch_init(cudaStream_t st, int nsm, u32 n, u64* best, u32 nwords, 
                         u64* acc, u32 nacc, u32* ctr, u32 nctr, u32* zero1, u32* ctr2, u32 nctr2);
 // weight threshold t of the light-edge phase: about `target` of the A records have w <= t
 // (binary search on a 4096-record sample); writes *t
-cudaError_t launch_light_threshold(cudaStream_t st, const uint4* arcs, u64 A, u64 target, u32* t);
+cudaError_t launch_light_threshold(cudaStream_t st, const uint4* arcs, u64 A, u64 target, u32* t,
+                                   u32 kfmt);
 // phi[x] = chain.m[len-1][...chain.m[0][x]] for x < n (-1 stays -1)
 cudaError_t launch_chain_compose(cudaStream_t st, int nsm, u32 n, const MapChain& chain, int* phi);
 // defer (light-edge phase): a component with no (light) edge left is kept, not finished
@@ -98,11 +99,25 @@ cudaError_t launch_filter_min(cudaStream_t st, int nsm, const u32* a_in, u64 a_m
 cudaError_t launch_uf_init(cudaStream_t st, int nsm, u32 n, u32* parent);
 cudaError_t launch_uf_pass(cudaStream_t st, int nsm, const u32* a_in, u64 a_max, const uint4* in,
                            u32* parent, uint4* out, u64* best, u32 n, u64* status, u32 epoch,
-                           u32* a_next, u32* tile_ctrs, u32& seq, const CompactCtl& cc, u32 s1,
+                           u32* a_next, u32* tile_ctrs, u32& seq, const CompactCtl& cc, u32 kfmt,
                            u64 tag);
-cudaError_t launch_uf_hook(cudaStream_t st, int nsm, u32 n, u32* parent, const u64* best, u32 s1,
+cudaError_t launch_uf_hook(cudaStream_t st, int nsm, u32 n, u32* parent, const u64* best, u32 kfmt,
                            bool tagged, u64 tag, const uint2* euv, u32* P, u32* msf, u64* acc,
                            u32* unions, const u32* surv, u64* hmap, u32 htag);
+// member-scan rounds (after the light-edge phase): *work += record ends of the vertices outside
+// the component of vertex 0 (phi: vertex -> component); member minima of those components
+// (own records [row[v] - wbase, row[v+1] - wbase) for owners in [vlo, vhi), reverse records
+// ridx[rrow[v] .. rrow[v+1])), best[phi[0]] = KEY_DEFER
+cudaError_t launch_member_work(cudaStream_t st, int nsm, u32 n, const int* phi, const u32* row,
+                               const u32* rrow, u32 vlo, u32 vhi, u64* work);
+cudaError_t launch_member_min(cudaStream_t st, int nsm, u32 n, const int* phi, const u32* row,
+                              const u32* rrow, const u32* ridx, const uint4* arcs, u32 vlo,
+                              u32 vhi, u32 wbase, u64* best, u32 kfmt);
+// the reverse index of the A local records (other endpoint -> record indices); rdeg, cursor:
+// n-word scratch; rrow: n + 1 words; ridx: A words
+cudaError_t launch_reverse_index(cudaStream_t st, int nsm, u32 n, u64 A, const uint4* arcs,
+                                 u32* rdeg, u32* rrow, u32* cursor, u32* ridx, u64* status,
+                                 u32 epoch);
 // kfmt: key format of the minima the pass emits = s1 | pb << 8 (pb = 0: (w << 32) | eid)
 cudaError_t launch_dense_best(cudaStream_t st, int nsm, u32 n, const u64* mat, u64* best);
 cudaError_t launch_dense_init(cudaStream_t st, int nsm, u32 n, u64* mat);

@@ -71,6 +71,8 @@ mst_status fail(mst_status s, const char* fmt, ...) {
         if (s_ != MST_OK) return s_;                                                      \
     } while (0)
 
+u32 bits_of(u64 x) { u32 b = 0; while (x) { ++b; x >>= 1; } return b; }
+
 // device-counter slots
 enum { C_ERR = 0, C_OUT = 1, C_NNEXT = 2, C_TILE = 3, C_AREC = 8 };  // C_TILE: 2 slots
 // C_AREC: per shard j and round r, the alive arcs entering round r (written by round r-1's
@@ -150,6 +152,9 @@ struct mst_graph {
     u64* xhost = nullptr;                // X_HOST: pinned staging (n + dense matrix entries)
     u64 xcap = 0;
     u64 A0_local = 0;                    // records built on this rank (all shards)
+    u32 vlo = 0, vhi = 0, wbase = 0;     // owners of this handle's records, their first record
+    u32 *rrow = nullptr, *ridx = nullptr;  // reverse index (member-scan rounds): other -> records
+    u64* mwork = nullptr;                // member-scan work estimate (device)
 
     bool opt_uf = false;     // MST_OPT_UNION_FIND (NEXT-3 variant)
     bool opt_small = true;   // MST_OPT_SMALL (one-CTA path for graphs that fit shared memory)
@@ -331,10 +336,21 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
         CK(cudaHostGetDevicePointer((void**)&g->dmap, hm, 0));
     }
 
-    CK(launch_degree(g->cst, g->nsm, (u32)n, (u32)m, src, dst, g->eu, g->ev, deg, g->dcnt + C_ERR));
+    CK(launch_degree(g->cst, g->nsm, (u32)n, (u32)m, src, dst, w, g->eu, g->ev, deg,
+                     g->dcnt + C_ERR, g->dcnt + C_WMAX));
     CK(cudaMemcpyAsync(g->hcnt, g->dcnt, sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
+    CK(cudaMemcpyAsync(g->hcnt + C_WMAX, g->dcnt + C_WMAX, sizeof(u32), cudaMemcpyDeviceToHost,
+                       g->cst));
     CK(cudaStreamSynchronize(g->cst));
     if (g->hcnt[0]) return fail(MST_EINVAL, "an endpoint is outside [0, n) (n = %lld)", (long long)n);
+    {   // packed minima keys when weight, edge id and a label fit in 63 bits (every handle:
+        // the keys' order is the (w, eid) order, so the MIN of a distributed run is unchanged);
+        // the records carry their key base, so the format is fixed before they are built
+        const u32 wb = bits_of(g->hcnt[C_WMAX]), eb = bits_of(m > 0 ? (u64)m - 1 : 0),
+                  pb = bits_of(n > 0 ? (u64)n - 1 : 0);
+        static const char* pk = getenv("MST_PACKED_KEYS");  // "0": always (w << 32) | eid
+        if (pb > 0 && wb + eb + pb <= 63 && !(pk && pk[0] == '0')) g->kfmt = (eb + pb) | (pb << 8);
+    }
 
     // owner degrees (each non-loop edge once, owned by one endpoint: owner_of())
     // default: the higher internal id (the lower-degree endpoint) owns the record, so the
@@ -391,7 +407,21 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CKS(galloc(g, &g->arcs0, A_loc));
     CKS(galloc(g, &g->euv, m));
     CK(launch_scatter(g->cst, g->nsm, (u32)m, g->eu, g->ev, w, cursor, g->arcs0, g->euv, hi_owner,
-                      g->dcnt + C_WMAX, (u32)vlo, (u32)vhi, (u32)wbase));
+                      g->kfmt, (u32)vlo, (u32)vhi, (u32)wbase));
+    g->vlo = (u32)vlo;
+    g->vhi = (u32)vhi;
+    g->wbase = (u32)wbase;
+    if (n > 0 && (u64)A0 >= 8ull * n) {
+        // heavy-tailed / dense inputs (the light-edge phase's regime): the reverse index of the
+        // records for the member-scan rounds (other endpoint -> record indices; build time only)
+        u32* rdeg;
+        CKS(galloc(g, &rdeg, n));
+        CKS(galloc(g, &g->rrow, n + 1));
+        CKS(galloc(g, &g->ridx, A_loc));
+        CKS(galloc(g, &g->mwork, 1));
+        CK(launch_reverse_index(g->cst, g->nsm, (u32)n, A_loc, g->arcs0, rdeg, g->rrow, cursor,
+                                g->ridx, g->status, g->epoch++));
+    }
     g->shards.clear();
     // light-edge phase: each shard's light records and their dead filler records (at most
     // LBLK_MAX per consumer warp of the pass) get their own window in abuf[0]
@@ -421,17 +451,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
         CKS(galloc(g, &g->mat[0], dense_entries(n)));
         CKS(galloc(g, &g->mat[1], dense_entries(n)));
     }
-    CK(cudaMemcpyAsync(g->hcnt + C_WMAX, g->dcnt + C_WMAX, sizeof(u32), cudaMemcpyDeviceToHost,
-                       g->cst));
     CK(cudaStreamSynchronize(g->cst));
-    {   // packed minima keys when weight, edge id and a label fit in 63 bits (every handle:
-        // the keys' order is the (w, eid) order, so the MIN of a distributed run is unchanged)
-        auto bits = [](u64 x) { u32 b = 0; while (x) { ++b; x >>= 1; } return b; };
-        const u32 wb = bits(g->hcnt[C_WMAX]), eb = bits(m > 0 ? (u64)m - 1 : 0),
-                  pb = bits(n > 0 ? (u64)n - 1 : 0);
-        static const char* pk = getenv("MST_PACKED_KEYS");  // "0": always (w << 32) | eid
-        if (pb > 0 && wb + eb + pb <= 63 && !(pk && pk[0] == '0')) g->kfmt = (eb + pb) | (pb << 8);
-    }
     g->st.n = g->n;
     g->st.m = g->m;
     g->st.arcs0 = (int64_t)g->A0;
@@ -594,15 +614,13 @@ void collect_profile(mst_graph* g) {
 // Graphs whose records, per-component arrays and forest bits fit one CTA's shared memory run
 // the whole method in one launch (kernels.cu k_small_msf): no per-round launches, no host
 // round trips (grid64: ~10 launches and a host wait per round for microseconds of work).
-u32 bits_of(u64 x) { u32 b = 0; while (x) { ++b; x >>= 1; } return b; }
 bool small_ok(const mst_graph* g) {
     static const char* e = getenv("MST_SMALL");  // "0": never (ablation)
     if (!g->opt_small || (e && e[0] == '0') || g->opt_keep || g->shards.size() != 1 ||
         g->xkind != X_NONE || g->n < 2)
         return false;
     const u64 E = g->shards[0].hi - g->shards[0].lo;
-    const u32 pb = bits_of((u64)g->n - 1), eb = bits_of(g->m > 0 ? (u64)g->m - 1 : 0);
-    return bits_of(g->hcnt[C_WMAX]) + eb + pb <= 64 &&
+    return g->kfmt != 0 &&  // (packed keys: the partner's label travels in the key)
            small_smem_bytes((u64)g->n, E, g->nwords) <= small_smem_limit();
 }
 struct SmallHost {  // (the layout of kernels.cu SmallOut)
@@ -614,11 +632,10 @@ mst_status run_small(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* ou
                      uint64_t* out_total, unsigned long long kl0) {
     static_assert(sizeof(SmallHost) == 8 + 8 + 512, "SmallOut layout");
     const u64 n = g->n, E = g->shards[0].hi - g->shards[0].lo;
-    const u32 pb = bits_of(n - 1), eb = bits_of(g->m > 0 ? (u64)g->m - 1 : 0);
     {
         Prof p(g, s, MST_K_SMALL, 0);
-        CK(launch_small(s, (u32)n, (u32)E, (u32)g->nwords, g->arcs0 + g->shards[0].lo, eb + pb, pb,
-                        out_ids, g->small_res));
+        CK(launch_small(s, (u32)n, (u32)E, (u32)g->nwords, g->arcs0 + g->shards[0].lo,
+                        g->kfmt & 0xffu, g->kfmt >> 8, out_ids, g->small_res));
     }
     CK(cudaMemcpyAsync(g->small_host, g->small_res, sizeof(SmallHost), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
@@ -666,11 +683,10 @@ mst_status run_uf(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out_n
         CK(cudaMemsetAsync(g->dcnt + C_UFU, 0, MST_MAX_ROUNDS * sizeof(u32), s));
     }
     // key format: tagged when weight and edge-id bits fit below the 6-bit round tag
-    auto bits = [](u64 x) { u32 b = 0; while (x) { ++b; x >>= 1; } return b; };
-    const u32 wb = bits(g->hcnt[C_WMAX]), eb = bits(g->m > 0 ? (u64)g->m - 1 : 0);
+    const u32 wb = bits_of(g->hcnt[C_WMAX]);
+    const u32 s1 = (g->kfmt >> 8) ? (g->kfmt & 0xffu) : 32u;  // the records' key format
     static const char* te = getenv("MST_UF_TAG");  // "0": untagged keys + a reset per round
-    const bool tagged = wb + eb <= 58 && !(te && te[0] == '0');
-    const u32 s1 = tagged ? eb : 32u;
+    const bool tagged = wb + s1 <= 58 && !(te && te[0] == '0');
     g->hcnt[arec(0, 0)] = sh.A = (u32)(sh.hi - sh.lo);
     CK(cudaMemcpyAsync(g->dcnt + arec(0, 0), g->hcnt + arec(0, 0), sizeof(u32),
                        cudaMemcpyHostToDevice, s));
@@ -707,11 +723,11 @@ mst_status run_uf(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out_n
             CK(launch_uf_pass(s, g->nsm, g->dcnt + arec(0, r), sh.hi - sh.lo, cur, parent,
                               never ? nullptr : const_cast<uint4*>(outbuf), g->bestA, (u32)n,
                               g->status, g->epoch++, g->dcnt + arec(0, r + 1), g->dcnt + C_TILE,
-                              g->pass_seq, cc, s1, tag));
+                              g->pass_seq, cc, g->kfmt, tag));
         }
         {
             Prof p(g, s, MST_K_HOOK, r);
-            CK(launch_uf_hook(s, g->nsm, (u32)n, parent, g->bestA, s1, tagged, tag, g->euv, g->P,
+            CK(launch_uf_hook(s, g->nsm, (u32)n, parent, g->bestA, g->kfmt, tagged, tag, g->euv, g->P,
                               g->msf, g->acc, g->dcnt + C_UFU + r, g->dcnt + C_SURV + r,
                               g->dmap + r, tag_base | (u32)r));
         }
@@ -786,6 +802,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     for (int r = 0; r < MST_MAX_ROUNDS; ++r) {
         g->st.n_r[r] = g->st.a_r[r] = 0;
         g->st.round_filter_ms[r] = 0;
+        g->st.member_ends[r] = -1;
     }
     if (n == 0) {
         *out_num = 0;
@@ -853,7 +870,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                 CK(cudaMemsetAsync(g->dcnt + C_LT, 0xff, sizeof(u32), s));
             else
                 CK(launch_light_threshold(s, g->arcs0, Al, (u64)((double)target * Al / g->A0),
-                                          g->dcnt + C_LT));
+                                          g->dcnt + C_LT, g->kfmt));
         }
         if (dist) {
             Prof p(g, s, MST_K_COMM, 0);
@@ -1072,15 +1089,52 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             CK(launch_dense_init(s, g->nsm, nn, g->mat[mc ^ 1]));
             CK(launch_dense_round(s, g->nsm, nr, g->mat[mc], Mr, nn, g->mat[mc ^ 1], bnxt));
         } else {
+            // member-scan round (after the light-edge phase): the records are read in vertex ids
+            // through Ψ; when the vertices outside the top hub's component own few record ends,
+            // their components' minima come from their members' records alone (kernels.cu)
+            bool member = false;
+            u64 mwork = 0;
+            static const char* me = getenv("MST_MEMBER_SCAN");  // "0": never (ablation)
+            if (phase == 2 && g->ridx && !(me && me[0] == '0') && cur == g->arcs0 && brnd == 0 &&
+                (phi_ready || brnd < r)) {
+                if (phi_ready) {  // (the switch composed the whole chain with M_r already)
+                } else {
+                    Prof p(g, s, MST_K_COMPOSE, r);
+                    CK(launch_compose(s, g->nsm, nb_sz, brnd == r - 1 ? chain.m[chain.len - 1] : g->phi,
+                                      Mr, g->phi));
+                    phi_ready = true;
+                }
+                {
+                    Prof p(g, s, MST_K_COMPOSE, r, 2);
+                    CK(cudaMemsetAsync(g->mwork, 0, sizeof(u64), s));
+                    CK(launch_member_work(s, g->nsm, (u32)n, g->phi, g->row, g->rrow, g->vlo, g->vhi,
+                                          g->mwork));
+                }
+                CK(cudaMemcpyAsync(&g->hacc[2 * ACC_SLOTS - 1], g->mwork, sizeof(u64),
+                                   cudaMemcpyDeviceToHost, s));
+                CK(cudaStreamSynchronize(s));
+                mwork = g->hacc[2 * ACC_SLOTS - 1];
+                if (dist) {  // the busiest rank decides for all (MAX = ~MIN(~x))
+                    u64 nx = ~mwork;
+                    CK(cudaMemcpyAsync(g->mwork, &nx, sizeof(u64), cudaMemcpyHostToDevice, s));
+                    CKS(xchg_min(g, s, g->mwork, 1, false));
+                    CK(cudaMemcpyAsync(&nx, g->mwork, sizeof(u64), cudaMemcpyDeviceToHost, s));
+                    CK(cudaStreamSynchronize(s));
+                    mwork = ~nx;
+                }
+                // record ends to touch, against the 2 E_0 of a pass over every record (random
+                // 16-B reads: worth it below ~1/16 of the streamed bytes)
+                member = mwork * 16 < 2 * g->A0 / (u64)std::max(1, g->nranks);
+            }
             // (light phase: only when its ~K n records outnumber the matrix cells — measured
             // on dense: 0.76 M light records against 5.7 M cells made the tail 2x slower)
-            to_dense = g->mat[0] && g->opt_dense && !g->opt_keep && nn <= (u32)DENSE_MAX &&
+            to_dense = !member && g->mat[0] && g->opt_dense && !g->opt_keep && nn <= (u32)DENSE_MAX &&
                        (phase != 1 || (u64)lk * n >= dense_entries(nn));
             if (to_dense) CK(launch_dense_init(s, g->nsm, nn, g->mat[0]));
             // A7: the map of this round's pass, from the records' label space (round brnd)
             // to round r+1: M_r itself, or composed over the rounds that did not compact
             const int* Mpass = Mr;
-            if (phi_ready) {  // (the switch composed the whole chain with M_r already)
+            if (phi_ready) {  // (the switch or the member decision composed Ψ with M_r already)
                 Mpass = g->phi;
                 phi_ready = false;
             } else if (brnd < r) {
@@ -1120,7 +1174,20 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                     cc.den = g->dcnt + C_SEEN + (r - 1);
                 }
             }
-            for (int j = 0; j < G; ++j) {
+            if (member) {
+                // the members' records of every component but the top hub's (deferred); the
+                // records themselves are untouched: the next full pass reads all of them
+                Prof p(g, s, MST_K_FILTER, r, MST_SUB_MEMBER);
+                CK(launch_member_min(s, g->nsm, (u32)n, g->phi, g->row, g->rrow, g->ridx, g->arcs0,
+                                     g->vlo, g->vhi, g->wbase, g->sim ? g->shard_best : bnxt, g->kfmt));
+                for (int j = 0; j < G; ++j) {
+                    g->hcnt[arec(j, r + 1)] = (u32)(g->shards[j].hi - g->shards[j].lo);
+                    CK(cudaMemcpyAsync(g->dcnt + arec(j, r + 1), g->hcnt + arec(j, r + 1),
+                                       sizeof(u32), cudaMemcpyHostToDevice, s));
+                }
+                g->st.member_ends[r] = (int64_t)mwork;
+            }
+            for (int j = 0; j < G && !member; ++j) {
                 Shard& sh = g->shards[j];
                 u64* tgt = g->sim ? g->shard_best + (u64)j * n : bnxt;
                 Prof p(g, s, MST_K_FILTER, r,
@@ -1144,7 +1211,9 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                                      g->kfmt));
             }
             if (to_dense && use_hub_row(g) && hub_ok) g->st.hub_row = 1;
-            if (adaptive) {
+            if (member) {
+                // (nothing compacted: the records stay in vertex ids, read through Ψ)
+            } else if (adaptive) {
                 pend = r;
                 pend_out = outbuf;
             } else if (!never && !to_dense) {

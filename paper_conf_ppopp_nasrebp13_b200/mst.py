@@ -24,7 +24,7 @@ KERNEL_NAMES = ["init", "min0", "hook", "jump", "filter", "output", "comm", "den
                 "compose", "small"]
 # launch sub-kinds per kind (include/mst.h MST_SUB_*)
 SUB_NAMES = {K_MIN0: ["min_all", "extract", "min_light"],
-             K_FILTER: ["sparse", "light", "switch", "transition"],
+             K_FILTER: ["sparse", "light", "switch", "transition", "member"],
              K_DENSE: ["dense_round", "dense_best", "tail"],
              K_COMPOSE: ["compose", "sample"]}
 
@@ -58,6 +58,7 @@ class mst_stats(ctypes.Structure):
         ("hub_row", ctypes.c_int32),
         ("light_switch_round", ctypes.c_int32),
         ("light_t", ctypes.c_uint32),
+        ("member_ends", ctypes.c_int64 * MAX_ROUNDS),
     ]
 
 
@@ -255,6 +256,7 @@ class MSTGraph:
             "hub_row": bool(s.hub_row),
             "light_switch_round": s.light_switch_round,
             "light_t": s.light_t,
+            "member_ends": list(s.member_ends[:R]),
         }
 
     def launch_times(self) -> list:

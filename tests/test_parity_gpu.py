@@ -609,3 +609,28 @@ def test_small_path_grid64_and_edges(lib, oracle_mod, gg):
     g = gg.config(2, scale_down=8)  # n = 16 K, m = 64 K
     st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, small=True)
     assert st["gpu_launches"] > 1
+
+
+# ------------------------------------------------------------------ member-scan rounds
+@pytest.mark.parametrize("k,sd,seed", [(4, 4, 1), (4, 2, 2), (4, 6, 3), (5, 6, 4)])
+def test_member_scan_rounds(lib, oracle_mod, gg, k, sd, seed):
+    """after the light-edge phase of a heavy-tailed graph the components outside the top hub's
+    take their minima from their members' records (reverse index) instead of a pass over every
+    record; the hub's component is deferred; bit-exact, re-runnable"""
+    g = gg.config(k, s=seed, scale_down=sd)
+    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, runs=2)
+    if k == 4 and st["light_switch_round"] >= 0:
+        assert any(x >= 0 for x in st["member_ends"])  # at least one member-scan round
+
+
+def test_member_scan_two_giants(lib, oracle_mod, gg):
+    """two heavy-tailed graphs side by side, joined by one heavy edge: after the light phase a
+    second giant lies outside the top hub's component, the member work is large, and the run
+    falls back to a pass over every record; bit-exact either way"""
+    a = gg.config(4, s=5, scale_down=4)
+    b = gg.config(4, s=6, scale_down=4)
+    n = a.n + b.n
+    src = np.concatenate([a.src, b.src + a.n, [0]]).astype(np.int32)
+    dst = np.concatenate([a.dst, b.dst + a.n, [a.n]]).astype(np.int32)
+    w = np.concatenate([a.w, b.w, [999]]).astype(np.uint32)
+    assert_parity(lib, oracle_mod, n, src, dst, w, runs=2)
