@@ -148,8 +148,10 @@ def byte_model(st):
         else:
             nxt_sparse = not (dr >= 0 and r + 1 >= dr)
             comp = st.get("compacted", [True] * R)[r]
+            din = st.get("dedup_in", [-1] * R)[r]
+            wrote = din if din >= 0 else a[r + 1]  # (A9: the pass wrote what the dedup then sorted)
             out.append({"kind": "filter", "compacted": bool(comp and nxt_sparse),
-                        "bytes": 16 * a[r] + (16 * a[r + 1] if (nxt_sparse and comp) else 0)})
+                        "bytes": 16 * a[r] + (16 * wrote if (nxt_sparse and comp) else 0)})
     return out
 
 
@@ -207,6 +209,8 @@ def run_gpu(args):
         h.set_option(mstb.mst.MST_OPT_KEEP_EDGES, 1)
     elif args.mode == "uf":
         h.set_option(mstb.mst.MST_OPT_UNION_FIND, 1)
+    elif args.mode == "dedup":
+        h.set_option(mstb.mst.MST_OPT_DEDUP, 1)
     if args.tau is not None:
         h.set_option(mstb.mst.MST_OPT_COMPACT_TAU, args.tau)
     build_ms = h.stats()["build_ms"]
@@ -438,10 +442,11 @@ def main():
                     choices=["grid64", "uniform", "road", "rmat22", "dense"])
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--mode", default="morph", choices=["morph", "sparse", "keep", "uf"],
+    ap.add_argument("--mode", default="morph", choices=["morph", "sparse", "keep", "uf", "dedup"],
                     help="morph: delete+compact, dense min-matrix at <= 4096 components "
                          "(default); sparse: never dense; keep: the paper's no-deletion scheme; "
-                         "uf: the union-find variant (NEXT-3)")
+                         "uf: the union-find variant (NEXT-3); dedup: A9 sort-based duplicate "
+                         "collapse after every sparse pass")
     ap.add_argument("--tau", type=int, default=None,
                     help="MST_OPT_COMPACT_TAU (permille; default: the library's)")
     ap.add_argument("--e2e-steps", type=int, default=3)

@@ -130,7 +130,8 @@ enum {
     MST_K_LIGHT = 8,   /* A2 light-edge threshold select (sampled radix select)       */
     MST_K_COMPOSE = 9, /* A7 label-map composition (+ the round-0 survival sample)    */
     MST_K_SMALL = 10,  /* A1-A11 in one CTA (MST_OPT_SMALL: graphs that fit smem)      */
-    MST_K_COUNT = 11
+    MST_K_DEDUP = 11,  /* A9 sort-based duplicate collapse (MST_OPT_DEDUP)            */
+    MST_K_COUNT = 12
 };
 /* launch sub-kinds (mst_launch_time.sub), so unlike launches of one kind are told apart:
  *   MST_K_MIN0  : MIN_ALL   = minima over every record (+ the light-record write);
@@ -178,6 +179,8 @@ typedef struct {
                                              0xffffffff when the phase was off            */
     int64_t member_ends[MST_MAX_ROUNDS];  /* member-scan round r: record ends read (the
                                              members' own + reverse records); -1: not one */
+    int64_t dedup_in[MST_MAX_ROUNDS];     /* A9: records entering the dedup after round r's
+                                             pass (a_r[r + 1] = after it); -1: none        */
 } mst_stats;
 
 mst_status mst_get_stats(const mst_graph* g, mst_stats* out);
@@ -247,12 +250,18 @@ mst_status mst_set_profiling(mst_graph* g, int enable);
  *       deletion, ascending ids): the latency regime of row A10, where the multi-kernel path
  *       pays launches and a host wait per round for microseconds of work. Single-GPU handles
  *       without MST_OPT_KEEP_EDGES / MST_OPT_UNION_FIND; 0 = always the multi-kernel path.
+ *   MST_OPT_DEDUP (default 0): 1 = row A9's sort-based duplicate collapse: after every
+ *       sparse pass (which then always compacts) the surviving records are sorted by their
+ *       component pair (CUB device radix sort) and each pair keeps its minimum key (CUB
+ *       reduce-by-key), leaving records grouped by their lower label (reading R13). Setting it
+ *       allocates ~32 B per local record of scratch (here, not in mst_run). Single-shard,
+ *       non-distributed handles; measured in DESIGN.md §5c. Never changes the result.
  * Keys of the component minima (rows A2/A8): (uint64(w) << 32) | eid, or, when the largest
  * weight, the largest edge id and the largest vertex id fit 63 bits together, the packed
  * (w << s1) | (eid << pb) | partner label — the same (w, eid) order (reading R17).
  */
 enum { MST_OPT_DENSE = 1, MST_OPT_KEEP_EDGES = 2, MST_OPT_DEVICE_TAIL = 3, MST_OPT_COMPACT_TAU = 4,
-       MST_OPT_LIGHT_FIRST = 5, MST_OPT_UNION_FIND = 6, MST_OPT_SMALL = 7 };
+       MST_OPT_LIGHT_FIRST = 5, MST_OPT_UNION_FIND = 6, MST_OPT_SMALL = 7, MST_OPT_DEDUP = 8 };
 mst_status mst_set_option(mst_graph* g, int option, int64_t value);
 
 /* ------------------------------------------------------------------ multi-GPU (§8(e))

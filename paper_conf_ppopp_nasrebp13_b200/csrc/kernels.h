@@ -44,6 +44,13 @@ cudaError_t launch_reorder(cudaStream_t st, int nsm, u32 n, u32 m, const u32* de
                            u32* eu, u32* ev, u32* newid, u32* counts, u64* status, u32 epoch,
                            u32* odeg, int hi_owner);
 u64 reorder_scratch(u64 n);
+// NEXT-4 BFS layout (MST_REORDER=2): newid = BFS discovery order from vertex `root` (then the
+// next unvisited vertex with an edge per component; edgeless vertices last), then the same
+// relabelling as launch_reorder. off: n + 1, cursor / q / newid: n, adj: 2 m, stt: 8 words.
+cudaError_t launch_reorder_bfs(cudaStream_t st, int nsm, u32 n, u32 m, const u32* deg, u32* degn,
+                               u32* eu, u32* ev, u32* off, u32* cursor, u32* adj, u32* q,
+                               u32* newid, u32* stt, u64* status, u32 epoch, u32* odeg,
+                               int hi_owner, u32 root);
 cudaError_t launch_owner_degree(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
                                 u32* odeg, int hi_owner);
 cudaError_t launch_scatter(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
@@ -118,6 +125,12 @@ cudaError_t launch_member_min(cudaStream_t st, int nsm, u32 n, const int* phi, c
 cudaError_t launch_reverse_index(cudaStream_t st, int nsm, u32 n, u64 A, const uint4* arcs,
                                  u32* rdeg, u32* rrow, u32* cursor, u32* ridx, u64* status,
                                  u32 epoch);
+// A9 (MST_OPT_DEDUP, dedup.cu): sort the A records {s', d', key base} in rec (labels < nlab) by
+// their pair (min, max) and keep the minimum key of every pair, in place; *a_count = records
+// left (written on the device). scratch: dedup_scratch_bytes(A) bytes; nruns: one device int
+size_t dedup_scratch_bytes(u64 A);
+cudaError_t launch_dedup(cudaStream_t st, int nsm, u64 A, u32 nlab, u32* a_count, uint4* rec,
+                         void* scratch, size_t scratch_bytes, int* nruns);
 // kfmt: key format of the minima the pass emits = s1 | pb << 8 (pb = 0: (w << 32) | eid)
 cudaError_t launch_dense_best(cudaStream_t st, int nsm, u32 n, const u64* mat, u64* best);
 cudaError_t launch_dense_init(cudaStream_t st, int nsm, u32 n, u64* mat);
@@ -129,6 +142,11 @@ cudaError_t launch_dense_tail(cudaStream_t st, int nsm, u32 n0, u64* best0, u64*
                               u32* msf, u64* acc, u32* bar, u32* stats, u64* trace = nullptr,
                               int defer = 0, int* map_out = nullptr, u32* n_out = nullptr);
 cudaError_t launch_compose(cudaStream_t st, int nsm, u32 nb, const int* src, const int* Mr, int* phi);
+// the same over vertex ids, also summing into *work the record ends of the vertices outside
+// the component *giant (the member-scan decision)
+cudaError_t launch_compose_work(cudaStream_t st, int nsm, u32 nb, const int* src, const int* Mr,
+                                int* phi, const int* giant, const u32* row, const u32* rrow,
+                                u32 vlo, u32 vhi, u64* work);
 cudaError_t launch_sample_survival(cudaStream_t st, const uint4* in, const u32* a_ptr, const int* M,
                                    u32* num, u32* den);
 // A10 latency regime: the whole method in one CTA (records, component arrays and forest bits

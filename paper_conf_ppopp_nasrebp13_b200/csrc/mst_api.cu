@@ -158,6 +158,10 @@ struct mst_graph {
 
     bool opt_uf = false;     // MST_OPT_UNION_FIND (NEXT-3 variant)
     bool opt_small = true;   // MST_OPT_SMALL (one-CTA path for graphs that fit shared memory)
+    bool opt_dedup = false;  // MST_OPT_DEDUP (A9: sort-based duplicate collapse after compaction)
+    void* dd_scratch = nullptr;  // its scratch (allocated when the option is set)
+    size_t dd_bytes = 0;
+    int* dd_runs = nullptr;
     void* small_res = nullptr;   // its device result block (SmallOut)
     void* small_host = nullptr;  // pinned copy
     bool opt_dense = true;   // MST_OPT_DENSE
@@ -358,8 +362,28 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     const char* op = getenv("MST_OWNER_MAX");
     const int hi_owner = (op && op[0] == '0') ? 0 : 1;
     CK(cudaMemsetAsync(cursor, 0, std::max<u64>(n, 1) * sizeof(u32), g->cst));
-    const char* ro = getenv("MST_REORDER");  // "0": keep the caller's vertex numbering
-    if (n > 0 && reorder && !(ro && ro[0] == '0')) {
+    const char* ro = getenv("MST_REORDER");  // "0": the caller's numbering, "2": BFS order
+    if (n > 0 && reorder && ro && ro[0] == '2') {
+        // NEXT-4 locality layout: BFS order from the highest-degree vertex (§6.1)
+        std::vector<u32> hd(n);
+        CK(cudaMemcpyAsync(hd.data(), deg, n * sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
+        CK(cudaStreamSynchronize(g->cst));
+        const u32 root = (u32)(std::max_element(hd.begin(), hd.end()) - hd.begin());
+        u32 *degn, *newid, *off, *bcur, *adj, *q, *stt;
+        CKS(galloc(g, &degn, n));
+        CKS(galloc(g, &newid, n));
+        CKS(galloc(g, &off, n + 1));
+        CKS(galloc(g, &bcur, n));
+        CKS(galloc(g, &adj, 2 * (u64)m));
+        CKS(galloc(g, &q, n));
+        CKS(galloc(g, &stt, 16));
+        CK(launch_reorder_bfs(g->cst, g->nsm, (u32)n, (u32)m, deg, degn, g->eu, g->ev, off, bcur,
+                              adj, q, newid, stt, g->status, g->epoch++, cursor, hi_owner, root));
+        u32 d0 = 0;
+        CK(cudaMemcpyAsync(&d0, degn, sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
+        CK(cudaStreamSynchronize(g->cst));
+        g->hub_row = (double)d0 * (double)n >= 16.0 * 2.0 * (double)m;
+    } else if (n > 0 && reorder && !(ro && ro[0] == '0')) {
         // A0 locality layout: hub-first internal numbering (stable, by log2 degree); the
         // relabelling pass also counts owner degrees in the new numbering
         u32 *degn, *newid, *counts;
@@ -803,6 +827,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         g->st.n_r[r] = g->st.a_r[r] = 0;
         g->st.round_filter_ms[r] = 0;
         g->st.member_ends[r] = -1;
+        g->st.dedup_in[r] = -1;
     }
     if (n == 0) {
         *out_num = 0;
@@ -954,6 +979,48 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         }
         pend = -1;
     };
+    // member-scan rounds (after the light-edge phase, kernels.cu "member-scan"): Ψ = vertex ->
+    // round r+1 label composed (if not yet) together with the record ends outside the top hub's
+    // component; the busiest rank's count decides for every rank
+    static const char* me_env = getenv("MST_MEMBER_SCAN");  // "0": never (ablation)
+    const bool member_ok = g->ridx && !(me_env && me_env[0] == '0');
+    auto member_work = [&](int rr, const int* Mrr, bool hubk, bool& ready, u64& work) -> mst_status {
+        CK(cudaMemsetAsync(g->mwork, 0, sizeof(u64), s));
+        if (!ready && hubk) {  // one pass: compose + count (the hub's label is tracked)
+            Prof p(g, s, MST_K_COMPOSE, rr, 2);
+            CK(launch_compose_work(s, g->nsm, (u32)n, rr >= 1 && chain.len ? (brnd == rr - 1 ? chain.m[chain.len - 1] : g->phi) : nullptr,
+                                   Mrr, g->phi, (const int*)g->dcnt + C_HUB + rr + 1, g->row,
+                                   g->rrow, g->vlo, g->vhi, g->mwork));
+        } else {
+            if (!ready) {
+                Prof p(g, s, MST_K_COMPOSE, rr);
+                CK(launch_compose(s, g->nsm, (u32)n, brnd == rr - 1 ? chain.m[chain.len - 1] : g->phi,
+                                  Mrr, g->phi));
+            }
+            Prof p(g, s, MST_K_COMPOSE, rr, 2);
+            CK(launch_member_work(s, g->nsm, (u32)n, g->phi, g->row, g->rrow, g->vlo, g->vhi,
+                                  g->mwork));
+        }
+        ready = true;
+        CK(cudaMemcpyAsync(&g->hacc[2 * ACC_SLOTS - 1], g->mwork, sizeof(u64),
+                           cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        work = g->hacc[2 * ACC_SLOTS - 1];
+        if (dist) {  // MAX over ranks = ~MIN(~x)
+            u64 nx = ~work;
+            CK(cudaMemcpyAsync(g->mwork, &nx, sizeof(u64), cudaMemcpyHostToDevice, s));
+            CKS(xchg_min(g, s, g->mwork, 1, false));
+            CK(cudaMemcpyAsync(&nx, g->mwork, sizeof(u64), cudaMemcpyDeviceToHost, s));
+            CK(cudaStreamSynchronize(s));
+            work = ~nx;
+        }
+        return MST_OK;
+    };
+    // record ends to touch against the 2 E_0 of a pass over every record (random 16-B reads:
+    // worth it below ~1/16 of the streamed bytes)
+    auto member_cheap = [&](u64 work) { return work * 16 < 2 * g->A0 / (u64)std::max(1, g->nranks); };
+    bool member_next = false;  // the phase-1 check chose a member-scan round for this round
+    u64 member_w = 0;
     bool dense = false;  // this round's alive arcs live in the min-matrix g->mat[mc]
     int mc = 0;
     g->st.dense_round = -1;
@@ -1053,8 +1120,25 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             ++r;
             break;
         }
-        static const u64 sw_den = getenv("MST_LIGHT_SWITCH") ? (u64)atoi(getenv("MST_LIGHT_SWITCH")) : 8;
-        if (phase == 1 && (was_v || nn == nr || (u64)(nr - nn) * sw_den < nr ||
+        // switch to all records when < 1/sw_den of the components merged: 1/8, or — when the
+        // member-scan rounds can take over (reverse index) — only once the light rounds stop
+        // merging: RMAT-22 merges 1.2 % in round 3 and 0.1 % in round 4, but those last merges
+        // join the big pieces of its giant (then the member scan finishes cheaply)
+        static const char* sw_env = getenv("MST_LIGHT_SWITCH");
+        const u64 sw_den = sw_env ? (u64)atoi(sw_env) : (member_ok ? (u64)n + 1 : 8);
+        member_next = false;
+        if (phase == 1 && member_ok && r >= 1 && !was_v && !dense && hub_ok && brnd == 0 &&
+            nn > 1 && (u64)(nr - nn) * 2 < nr && moff + nr + 3ull * nn <= 3 * n) {
+            // light phase: once only the top hub's component is big (the others own few record
+            // ends), a member-scan round replaces both the next light pass and the pass over
+            // every record (RMAT-22: ~10 K small components, 2.37 M vertices in the giant)
+            CKS(member_work(r, Mr, true, phi_ready, member_w));
+            member_next = member_cheap(member_w);
+            static const bool dbg1 = getenv("MST_DEBUG_MEMBER") != nullptr;
+            if (dbg1) fprintf(stderr, "light round %d: nr %u nn %u member work %llu -> %d\n", r, nr,
+                              nn, (unsigned long long)member_w, (int)member_next);
+        }
+        if (phase == 1 && (member_next || was_v || nn == nr || (u64)(nr - nn) * sw_den < nr ||
                            moff + nr + 3ull * nn > 3 * n)) {
             // no light edge joins two components any more (every component would otherwise
             // have merged or absorbed one), or < 1/8 merged (most components are deferred:
@@ -1064,7 +1148,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             phase = 2;
             dense = false;  // the records are read again (a dense phase-1 matrix is dropped)
             g->st.light_switch_round = r;
-            if (r >= 1 && chain.len + 1 < MST_CHAIN_MAX) {  // Ψ = Mr ∘ chain in one kernel
+            if (!phi_ready && r >= 1 && chain.len + 1 < MST_CHAIN_MAX) {  // Ψ = Mr ∘ chain in one kernel
                 Prof p(g, s, MST_K_COMPOSE, r);
                 MapChain full = chain;
                 full.m[full.len++] = Mr;
@@ -1093,38 +1177,41 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             // through Ψ; when the vertices outside the top hub's component own few record ends,
             // their components' minima come from their members' records alone (kernels.cu)
             bool member = false;
-            u64 mwork = 0;
-            static const char* me = getenv("MST_MEMBER_SCAN");  // "0": never (ablation)
-            if (phase == 2 && g->ridx && !(me && me[0] == '0') && cur == g->arcs0 && brnd == 0 &&
-                (phi_ready || brnd < r)) {
-                if (phi_ready) {  // (the switch composed the whole chain with M_r already)
-                } else {
-                    Prof p(g, s, MST_K_COMPOSE, r);
-                    CK(launch_compose(s, g->nsm, nb_sz, brnd == r - 1 ? chain.m[chain.len - 1] : g->phi,
-                                      Mr, g->phi));
-                    phi_ready = true;
+            u64 mwork = member_w;
+            if (member_next) {
+                member = true;  // (decided by the phase-1 check of this round)
+            } else if (phase == 2 && member_ok && cur == g->arcs0 && brnd == 0 &&
+                       (phi_ready || brnd < r)) {
+                CKS(member_work(r, Mr, hub_ok, phi_ready, mwork));
+                member = member_cheap(mwork);
+                static const bool dbg = getenv("MST_DEBUG_MEMBER") != nullptr;
+                if (dbg) {
+                    fprintf(stderr, "member round %d: nn %u work %llu A0 %llu -> %d\n", r, nn,
+                            (unsigned long long)mwork, (unsigned long long)g->A0, (int)member);
+                    std::vector<int> ph(n);
+                    std::vector<u32> rw(n + 1), rr(n + 1);
+                    CK(cudaMemcpy(ph.data(), g->phi, n * 4, cudaMemcpyDeviceToHost));
+                    CK(cudaMemcpy(rw.data(), g->row, (n + 1) * 4, cudaMemcpyDeviceToHost));
+                    CK(cudaMemcpy(rr.data(), g->rrow, (n + 1) * 4, cudaMemcpyDeviceToHost));
+                    std::vector<u64> sz(nn + 1, 0), dg(nn + 1, 0);
+                    u64 fin = 0;
+                    for (u64 v = 0; v < n; ++v) {
+                        if (ph[v] < 0) { ++fin; continue; }
+                        sz[ph[v]]++;
+                        dg[ph[v]] += (rw[v + 1] - rw[v]) + (rr[v + 1] - rr[v]);
+                    }
+                    u64 big = 0;
+                    for (u32 c = 0; c < nn; ++c) if (sz[c] > sz[big]) big = c;
+                    if (FILE* f = fopen("gpurun_out/phi.bin", "wb")) {
+                        fwrite(ph.data(), 4, n, f);
+                        fclose(f);
+                    }
+                    fprintf(stderr, "  phi[0] = %d (size %llu, ends %llu); largest comp %llu size %llu ends %llu; finished vertices %llu; rrow[n] %u row[n] %u\n",
+                            ph[0], ph[0] >= 0 ? (unsigned long long)sz[ph[0]] : 0ull,
+                            ph[0] >= 0 ? (unsigned long long)dg[ph[0]] : 0ull, (unsigned long long)big,
+                            (unsigned long long)sz[big], (unsigned long long)dg[big], (unsigned long long)fin,
+                            rr[n], rw[n]);
                 }
-                {
-                    Prof p(g, s, MST_K_COMPOSE, r, 2);
-                    CK(cudaMemsetAsync(g->mwork, 0, sizeof(u64), s));
-                    CK(launch_member_work(s, g->nsm, (u32)n, g->phi, g->row, g->rrow, g->vlo, g->vhi,
-                                          g->mwork));
-                }
-                CK(cudaMemcpyAsync(&g->hacc[2 * ACC_SLOTS - 1], g->mwork, sizeof(u64),
-                                   cudaMemcpyDeviceToHost, s));
-                CK(cudaStreamSynchronize(s));
-                mwork = g->hacc[2 * ACC_SLOTS - 1];
-                if (dist) {  // the busiest rank decides for all (MAX = ~MIN(~x))
-                    u64 nx = ~mwork;
-                    CK(cudaMemcpyAsync(g->mwork, &nx, sizeof(u64), cudaMemcpyHostToDevice, s));
-                    CKS(xchg_min(g, s, g->mwork, 1, false));
-                    CK(cudaMemcpyAsync(&nx, g->mwork, sizeof(u64), cudaMemcpyDeviceToHost, s));
-                    CK(cudaStreamSynchronize(s));
-                    mwork = ~nx;
-                }
-                // record ends to touch, against the 2 E_0 of a pass over every record (random
-                // 16-B reads: worth it below ~1/16 of the streamed bytes)
-                member = mwork * 16 < 2 * g->A0 / (u64)std::max(1, g->nranks);
             }
             // (light phase: only when its ~K n records outnumber the matrix cells — measured
             // on dense: 0.76 M light records against 5.7 M cells made the tail 2x slower)
@@ -1155,7 +1242,10 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             int dsh = -1;  // the shard whose pass reports the device-side decision
             for (int j = 0; j < G && dsh < 0; ++j)
                 if (g->shards[j].hi > g->shards[j].lo) dsh = j;
-            const bool adaptive = !to_dense && !never && g->tau < 1000 && dsh >= 0;
+            // (A9 dedup needs the survivors compacted: it always compacts then)
+            const bool dedup = g->opt_dedup && g->dd_scratch && G == 1 && !dist && !to_dense &&
+                               !never && !member && phase != 1;
+            const bool adaptive = !to_dense && !never && g->tau < 1000 && dsh >= 0 && !dedup;
             const uint4* outbuf = (cur == g->abuf[0]) ? g->abuf[1] : g->abuf[0];
             CompactCtl cc;
             cc.surv = g->dcnt + C_SURV + r;
@@ -1217,6 +1307,17 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                 pend = r;
                 pend_out = outbuf;
             } else if (!never && !to_dense) {
+                if (dedup) {  // A9: sort the survivors by component pair, keep each pair's minimum
+                    u32 acnt = 0;
+                    CK(cudaMemcpyAsync(&acnt, g->dcnt + arec(0, r + 1), sizeof(u32),
+                                       cudaMemcpyDeviceToHost, s));
+                    CK(cudaStreamSynchronize(s));
+                    g->st.dedup_in[r] = acnt;
+                    Prof p(g, s, MST_K_DEDUP, r);
+                    CK(launch_dedup(s, g->nsm, acnt, nn, g->dcnt + arec(0, r + 1),
+                                    const_cast<uint4*>(outbuf) + g->shards[0].lo, g->dd_scratch,
+                                    g->dd_bytes, g->dd_runs));
+                }
                 cur = outbuf;
                 cur_light = false;
                 brnd = r + 1;
@@ -1518,6 +1619,15 @@ mst_status mst_set_option(mst_graph* g, int option, int64_t value) {
             g->opt_uf = value != 0;
         } else if (option == MST_OPT_SMALL) {
             g->opt_small = value != 0;
+        } else if (option == MST_OPT_DEDUP) {
+            g->opt_dedup = value != 0;
+            if (g->opt_dedup && !g->dd_scratch) {  // (allocated here: mst_run allocates nothing)
+                const u64 A = std::max<u64>(g->A0_local, 1);
+                g->dd_bytes = dedup_scratch_bytes(A);
+                CKS(galloc(g, reinterpret_cast<unsigned char**>(&g->dd_scratch), g->dd_bytes));
+                CKS(galloc(g, &g->dd_runs, 2));
+                CK(cudaStreamSynchronize(g->cst));
+            }
         } else {
             return fail(MST_EINVAL, "unknown option %d", option);
         }

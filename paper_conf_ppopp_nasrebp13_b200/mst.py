@@ -19,9 +19,9 @@ STATUS_NAMES = {0: "MST_OK", 1: "MST_EINVAL", 2: "MST_ENOMEM", 3: "MST_ECUDA", 4
                 5: "MST_EINTERNAL", 6: "MST_ENOTSUP"}
 MAX_ROUNDS = 64
 K_INIT, K_MIN0, K_HOOK, K_JUMP, K_FILTER, K_OUTPUT, K_COMM, K_DENSE, K_LIGHT, K_COMPOSE, \
-    K_SMALL, K_COUNT = range(12)
+    K_SMALL, K_DEDUP, K_COUNT = range(13)
 KERNEL_NAMES = ["init", "min0", "hook", "jump", "filter", "output", "comm", "dense", "light",
-                "compose", "small"]
+                "compose", "small", "dedup"]
 # launch sub-kinds per kind (include/mst.h MST_SUB_*)
 SUB_NAMES = {K_MIN0: ["min_all", "extract", "min_light"],
              K_FILTER: ["sparse", "light", "switch", "transition", "member"],
@@ -39,6 +39,7 @@ MST_OPT_DENSE, MST_OPT_KEEP_EDGES, MST_OPT_DEVICE_TAIL, MST_OPT_COMPACT_TAU = 1,
 MST_OPT_LIGHT_FIRST = 5
 MST_OPT_UNION_FIND = 6
 MST_OPT_SMALL = 7
+MST_OPT_DEDUP = 8
 
 
 class mst_stats(ctypes.Structure):
@@ -59,6 +60,7 @@ class mst_stats(ctypes.Structure):
         ("light_switch_round", ctypes.c_int32),
         ("light_t", ctypes.c_uint32),
         ("member_ends", ctypes.c_int64 * MAX_ROUNDS),
+        ("dedup_in", ctypes.c_int64 * MAX_ROUNDS),
     ]
 
 
@@ -257,6 +259,7 @@ class MSTGraph:
             "light_switch_round": s.light_switch_round,
             "light_t": s.light_t,
             "member_ends": list(s.member_ends[:R]),
+            "dedup_in": list(s.dedup_in[:R]),
         }
 
     def launch_times(self) -> list:

@@ -26,6 +26,7 @@ KNOBS = [
     {"MST_QFILTER": "0"},        # no quantised-weight filter
     {"MST_QFILTER": "2"},        # filter tables in every filter pass
     {"MST_REORDER": "0"},        # caller's vertex numbering (no hub-first layout)
+    {"MST_REORDER": "2"},        # BFS-order layout (NEXT-4)
     {"MST_PACKED_KEYS": "0"},    # always (w << 32) | eid keys
     {"MST_OWNER_MAX": "0"},      # lower internal id owns each record
     {"MST_HUB_ROW": "0"},

@@ -634,3 +634,30 @@ def test_member_scan_two_giants(lib, oracle_mod, gg):
     dst = np.concatenate([a.dst, b.dst + a.n, [a.n]]).astype(np.int32)
     w = np.concatenate([a.w, b.w, [999]]).astype(np.uint32)
     assert_parity(lib, oracle_mod, n, src, dst, w, runs=2)
+
+
+# ------------------------------------------------------------------ A9: sort-based dedup
+DEDUP = 8  # MST_OPT_DEDUP (include/mst.h)
+
+
+@pytest.mark.parametrize("k,sd", [(2, 6), (3, 8), (4, 6), (5, 6), (2, 2)])
+def test_dedup_configs(lib, oracle_mod, gg, k, sd):
+    """after every sparse pass the survivors are sorted by component pair and only each pair's
+    minimum record is kept (A9); the forest is unchanged and the records shrink"""
+    g = gg.config(k, s=11, scale_down=sd)
+    for extra in ([], [(lib.mst.MST_OPT_DENSE, 0), (LF, 0)]):
+        st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w, runs=2,
+                           options=[(DEDUP, 1)] + extra)
+        for r, din in enumerate(st["dedup_in"]):
+            if din >= 0:
+                assert st["a_r"][r + 1] <= din  # never more records after the dedup
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_dedup_random_multigraphs(lib, oracle_mod, seed):
+    rng = np.random.default_rng(6100 + seed)
+    n = int(rng.integers(2, 30_000))
+    m = int(rng.integers(0, 40 * n))
+    src, dst, w = mc.random_multigraph(rng, n, m, [1, 7, 1000, 2**32 - 1][seed % 4])
+    assert_parity(lib, oracle_mod, n, src, dst, w, runs=2,
+                  options=[(DEDUP, 1), (lib.mst.MST_OPT_DENSE, seed % 2)])

@@ -11,7 +11,7 @@ try:
     d = json.load(open(f"/tmp/ab_{v}.json"))
     lk = d.get("launch_kinds", {})
     ks = " ".join(f"{k}={x['ms_per_step']*1e3:.0f}" for k, x in lk.items() if x["ms_per_step"] > 0.02)
-    print(f"[{v:10s}] {wl:7s} {d['value']/1e9:7.3f} G/s {d['ms_per_step']:.4f} ms  frac {d['roofline']['frac']:.3f}  {d['parity']}  {ks}")
+    print(f"[{v:10s}] {wl:7s} {d['value']/1e9:7.3f} G/s {d['ms_per_step']:.4f} ms  frac {d['roofline']['frac'] or 0:.3f}  {d['parity']}  {ks}")
 except Exception as e:
     print(f"[{v}] {wl} failed: {e}", open(f"/tmp/ab_{v}.err").read()[-600:])
 PY

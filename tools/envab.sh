@@ -12,7 +12,7 @@ try:
     lk = d.get("launch_kinds", {})
     ks = " ".join(f"{k}={x['ms_per_step']*1e3:.0f}" for k, x in lk.items() if x["ms_per_step"] > 0.02)
     rs = " ".join(f"r{r['r']}:{r['n_r']}" for r in d["rounds"])
-    print(f"[{g:24s}] {wl:7s} {d['value']/1e9:7.3f} G/s {d['ms_per_step']:.4f} ms  frac {d['roofline']['frac']:.3f}  {ks}  | {rs}")
+    print(f"[{g:24s}] {wl:7s} {d['value']/1e9:7.3f} G/s {d['ms_per_step']:.4f} ms  frac {d['roofline']['frac'] or 0:.3f}  {ks}  | {rs}")
 except Exception as e:
     print(f"[{g}] {wl} failed: {e}", open("/tmp/eab.err").read()[-600:])
 PY
