@@ -871,6 +871,9 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                  g->A0 >= 4ull * lk * n) ? 1 : 0;  // light records <= a quarter
     const bool dist = g->xkind != X_NONE;
     const bool light_only0 = lo0_want && phase;
+    // member-scan rounds can finish the light phase (reverse index built: >= 8 records/vertex)
+    static const char* me_env = getenv("MST_MEMBER_SCAN");  // "0": never (ablation)
+    const bool member_ok = g->ridx && !(me_env && me_env[0] == '0');
     g->st.light_switch_round = -1;
     g->st.light_t = 0xffffffffu;
     if (phase) {
@@ -885,8 +888,12 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             // edges/s) while t 120-150 is flat; the 4096-record sample puts t within ~+-5
             // (dense regime, K = 8: aimed at 10 n so that t <= 2 — light degree ~8, a few
             // vertices without a light edge and one more all-records pass — stays unlikely)
+            // (with member-scan rounds, fewer light records pay: the components the light
+            // phase leaves are finished by member scans, not by a pass over every record;
+            // measured on RMAT-22: t 139 -> 60, 62.8 -> 66.1 G edges/s; t 40: 64.9)
             const bool auto_k = lk_env == 0xffffffffu && g->light_k < 0;
-            const u64 target = !auto_k ? (u64)lk * n : lo0_want ? (u64)10 * n : (u64)23 * n / 10;
+            const u64 target = !auto_k ? (u64)lk * n : lo0_want ? (u64)10 * n
+                             : member_ok ? (u64)n : (u64)23 * n / 10;
             // a rank samples its own records, aimed at the same fraction of them; every rank
             // must use the SAME t (a mixed threshold is not a prefix of the (w, id) order),
             // so the ranks agree on the smallest sampled t
@@ -982,8 +989,6 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     // member-scan rounds (after the light-edge phase, kernels.cu "member-scan"): Ψ = vertex ->
     // round r+1 label composed (if not yet) together with the record ends outside the top hub's
     // component; the busiest rank's count decides for every rank
-    static const char* me_env = getenv("MST_MEMBER_SCAN");  // "0": never (ablation)
-    const bool member_ok = g->ridx && !(me_env && me_env[0] == '0');
     auto member_work = [&](int rr, const int* Mrr, bool hubk, bool& ready, u64& work) -> mst_status {
         CK(cudaMemsetAsync(g->mwork, 0, sizeof(u64), s));
         if (!ready && hubk) {  // one pass: compose + count (the hub's label is tracked)

@@ -242,7 +242,10 @@ def test_profiling_stats(lib, gg):
 @pytest.mark.parametrize("k", [1, 2, 3, 4, 5])
 def test_full_size_configs(lib, oracle_mod, gg, k):
     g = gg.config(k)
-    assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w)
+    st = assert_parity(lib, oracle_mod, g.n, g.src, g.dst, g.w)
+    # |F| = n - c with c from the oracle's own component labelling (not from Kruskal)
+    _, c = oracle_mod.components(g.n, g.src, g.dst)
+    assert st["num_edges"] == g.n - c
 
 
 # ------------------------------------------------------------------ sparse-only rounds

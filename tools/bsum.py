@@ -17,4 +17,5 @@ for p in sys.argv[1:]:
               f"{v['ms_per_step']*1e3:8.1f} us/step  frac {v['frac'] or 0:.3f}")
     for r in d.get("rounds", []):
         print(f"   r{r['r']} {r['kind']:9s} n={r['n_r']:>9} A={r['A_r']:>10} comp={r['compacted']} "
-              f"{r['filter_ms']*1e3:7.1f} us frac {r['frac'] or 0:.3f}")
+              f"{r['filter_ms']*1e3:7.1f} us frac {r['frac'] or 0:.3f}  hook {r.get('hook_ms', 0)*1e3:6.1f} "
+              f"jump {r.get('jump_ms', 0)*1e3:6.1f} compose {r.get('compose_ms', 0)*1e3:6.1f} us")
