@@ -354,7 +354,7 @@ def run_gpu(args):
                        "generator": "graphgen (SURVEY.md §8(d) recipe)",
                        "l2": "flushed between timed steps (256 MB write); arcs > L2",
                        "parallelism": f"edge-sharded x{world}" if world > 1 else "1 GPU",
-                       "build_ms": build_ms, "gen_s": gen_s},
+                       "build_ms": build_ms, "gen_s": gen_s, "layout": st.get("layout")},
             "parity": parity,
             "num_edges": cnt, "total_weight": tot,
             # the dominant kernel of the step (largest share): the per-round pass (A8) or the

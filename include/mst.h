@@ -181,6 +181,8 @@ typedef struct {
                                              members' own + reverse records); -1: not one */
     int64_t dedup_in[MST_MAX_ROUNDS];     /* A9: records entering the dedup after round r's
                                              pass (a_r[r + 1] = after it); -1: none        */
+    int32_t layout;                       /* internal vertex numbering of the build: 0 the
+                                             caller's, 1 hub-first, 2 BFS order (NEXT-4)   */
 } mst_stats;
 
 mst_status mst_get_stats(const mst_graph* g, mst_stats* out);

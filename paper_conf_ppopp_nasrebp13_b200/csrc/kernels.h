@@ -37,7 +37,8 @@ struct CompactCtl {
 };
 
 cudaError_t launch_degree(cudaStream_t st, int nsm, u32 n, u32 m, const int* src, const int* dst,
-                          const unsigned* w, u32* eu, u32* ev, u32* deg, u32* err, u32* wmax);
+                          const unsigned* w, u32* eu, u32* ev, u32* deg, u32* err, u32* wmax,
+                          u64* span);  // *span += sum over non-loop edges of |u - v|
 cudaError_t launch_scan_rows(cudaStream_t st, u32 n, const u32* deg, u32* row, u32* cursor,
                              u64* status, u32 epoch);
 cudaError_t launch_reorder(cudaStream_t st, int nsm, u32 n, u32 m, const u32* deg, u32* degn,

@@ -340,8 +340,13 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
         CK(cudaHostGetDevicePointer((void**)&g->dmap, hm, 0));
     }
 
+    u64* dspan;
+    CKS(galloc(g, &dspan, 1));
+    CK(cudaMemsetAsync(dspan, 0, sizeof(u64), g->cst));
     CK(launch_degree(g->cst, g->nsm, (u32)n, (u32)m, src, dst, w, g->eu, g->ev, deg,
-                     g->dcnt + C_ERR, g->dcnt + C_WMAX));
+                     g->dcnt + C_ERR, g->dcnt + C_WMAX, dspan));
+    u64 span = 0;
+    CK(cudaMemcpyAsync(&span, dspan, sizeof(u64), cudaMemcpyDeviceToHost, g->cst));
     CK(cudaMemcpyAsync(g->hcnt, g->dcnt, sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
     CK(cudaMemcpyAsync(g->hcnt + C_WMAX, g->dcnt + C_WMAX, sizeof(u32), cudaMemcpyDeviceToHost,
                        g->cst));
@@ -362,12 +367,29 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     const char* op = getenv("MST_OWNER_MAX");
     const int hi_owner = (op && op[0] == '0') ? 0 : 1;
     CK(cudaMemsetAsync(cursor, 0, std::max<u64>(n, 1) * sizeof(u32), g->cst));
-    const char* ro = getenv("MST_REORDER");  // "0": the caller's numbering, "2": BFS order
-    if (n > 0 && reorder && ro && ro[0] == '2') {
-        // NEXT-4 locality layout: BFS order from the highest-degree vertex (PAPER.md §6.1 L231)
-        std::vector<u32> hd(n);
+    const char* ro = getenv("MST_REORDER");  // "0": the caller's numbering, "1": hub-first, "2": BFS
+    std::vector<u32> hd;
+    bool bfs = ro && ro[0] == '2';
+    if (n > 0 && reorder && !ro) {
+        // auto layout (NEXT-4, measured in DESIGN.md §5d): heavy-tailed degrees -> hub-first;
+        // near-regular degrees whose ids carry no locality (mean |u - v| > n / 8: uniform,
+        // dense) -> BFS order; near-regular with local ids (road, grids) -> hub-first, i.e.
+        // the caller's order within equal degree buckets
+        hd.resize(n);
         CK(cudaMemcpyAsync(hd.data(), deg, n * sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
         CK(cudaStreamSynchronize(g->cst));
+        const u32 dmax = *std::max_element(hd.begin(), hd.end());
+        const bool heavy = (double)dmax * (double)n >= 16.0 * 2.0 * (double)m;
+        bfs = !heavy && m > 0 && (double)span / (double)m > (double)n / 8.0;
+    }
+    g->st.layout = (n > 0 && reorder && !(ro && ro[0] == '0')) ? (bfs ? 2 : 1) : 0;
+    if (n > 0 && reorder && bfs) {
+        // NEXT-4 locality layout: BFS order from the highest-degree vertex (PAPER.md §6.1 L231)
+        if (hd.empty()) {
+            hd.resize(n);
+            CK(cudaMemcpyAsync(hd.data(), deg, n * sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
+            CK(cudaStreamSynchronize(g->cst));
+        }
         const u32 root = (u32)(std::max_element(hd.begin(), hd.end()) - hd.begin());
         u32 *degn, *newid, *off, *bcur, *adj, *q, *stt;
         CKS(galloc(g, &degn, n));

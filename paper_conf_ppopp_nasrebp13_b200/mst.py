@@ -61,6 +61,7 @@ class mst_stats(ctypes.Structure):
         ("light_t", ctypes.c_uint32),
         ("member_ends", ctypes.c_int64 * MAX_ROUNDS),
         ("dedup_in", ctypes.c_int64 * MAX_ROUNDS),
+        ("layout", ctypes.c_int32),
     ]
 
 
@@ -260,6 +261,7 @@ class MSTGraph:
             "light_t": s.light_t,
             "member_ends": list(s.member_ends[:R]),
             "dedup_in": list(s.dedup_in[:R]),
+            "layout": ["caller", "hub-first", "bfs"][s.layout] if 0 <= s.layout < 3 else s.layout,
         }
 
     def launch_times(self) -> list:
