@@ -334,11 +334,17 @@ def run_gpu(args):
                     "frac": a / peak if a else None, "peak_source": peak_src,
                     "avg_launch_ms": ms / max(launches, 1), "bytes_per_launch": byts / max(launches, 1),
                     "share_of_step": ms / step_prof if step_prof else None}
+        # the one-CTA path (graphs that fit shared memory): the whole run is one launch,
+        # latency-bound; its algorithmic bytes are the records read once + the ids written
+        sm = by_kind.get(("small", "0"))
+        small_ms = sm[1] if sm else 0.0
+        dom = "small" if small_ms > max(filt_ms, min0_ms) else ("A8" if filt_ms >= min0_ms else "A2")
         traffic = None
         tp = os.path.join(ROOT, "profiles", f"ncu_traffic_{args.workload}.json")
         if os.path.exists(tp):
-            traffic = json.load(open(tp)).get(
-                "filter_dram_bytes_per_launch" if filt_ms >= min0_ms else "min0_dram_bytes_per_launch")
+            traffic = json.load(open(tp)).get({"A8": "filter_dram_bytes_per_launch",
+                                               "A2": "min0_dram_bytes_per_launch",
+                                               "small": "small_dram_bytes_per_launch"}[dom])
         rounds = []
         for rr in round_acc or []:
             gbs = rr["filter_bytes"] / (rr["filter_ms"] * 1e-3) / 1e9 if rr["filter_ms"] > 0 else None
@@ -360,10 +366,12 @@ def run_gpu(args):
             # the dominant kernel of the step (largest share): the per-round pass (A8) or the
             # round-0 minimum (A2, which also writes the light records when that phase is on)
             "roofline": {**(kernel_roof("k_arc_pass<MODE_FILTER> (A8)", filt_ms, filt_bytes,
-                                        filt_launches)
-                            if filt_ms >= min0_ms else
+                                        filt_launches) if dom == "A8" else
                             kernel_roof("k_arc_pass<MODE_MIN0> (A2)", min0_ms, min0_bytes,
-                                        min0_launches)),
+                                        min0_launches) if dom == "A2" else
+                            {**kernel_roof("k_small_msf (A1-A11, one CTA)", small_ms,
+                                           (16 * st["arcs0"] + 4 * cnt) * args.steps, sm[0]),
+                             "bound": "latency"}),
                          "traffic": traffic,
                          "timing": "CUDA events around every launch on the run's stream, "
                                    "over a second timed region of the same K steps (value "

@@ -99,7 +99,8 @@ cudaError_t launch_filter_min(cudaStream_t st, int nsm, const u32* a_in, u64 a_m
                               const uint4* in, const int* M, uint4* out, u64* best, u32 nb,
                               u64* status, u32 epoch, u32* a_next, u32* tile_ctrs, u32& seq,
                               u64* mat, const CompactCtl& cc = CompactCtl(),
-                              const int* hub = nullptr, u32 kfmt = 0);
+                              const int* hub = nullptr, u32 kfmt = 0, bool adj = false);
+// adj: A8's adjacent-duplicate filter in a compacting pass
 // NEXT-3 union-find variant: parent = identity; one pass (K1: roots by find,
 // intra-component records dropped, survivors compacted unchanged when the policy says so,
 // minima keys (w << s1 | eid) | tag into best[root]); then partner + union (K2a/K2b: forest
@@ -108,7 +109,7 @@ cudaError_t launch_uf_init(cudaStream_t st, int nsm, u32 n, u32* parent);
 cudaError_t launch_uf_pass(cudaStream_t st, int nsm, const u32* a_in, u64 a_max, const uint4* in,
                            u32* parent, uint4* out, u64* best, u32 n, u64* status, u32 epoch,
                            u32* a_next, u32* tile_ctrs, u32& seq, const CompactCtl& cc, u32 kfmt,
-                           u64 tag);
+                           u64 tag, bool adj = false);
 cudaError_t launch_uf_hook(cudaStream_t st, int nsm, u32 n, u32* parent, const u64* best, u32 kfmt,
                            bool tagged, u64 tag, const uint2* euv, u32* P, u32* msf, u64* acc,
                            u32* unions, const u32* surv, u64* hmap, u32 htag);
@@ -153,12 +154,12 @@ cudaError_t launch_sample_survival(cudaStream_t st, const uint4* in, const u32* 
 // A10 latency regime: the whole method in one CTA (records, component arrays and forest bits
 // in shared memory) when small_smem_bytes(n, E, nwords) <= small_smem_limit() and packed keys
 // (w << s1 | eid << pb | partner) fit 64 bits; res (device, small_out_bytes()) receives
-// {count, rounds, total, n_r[64], a_r[64]}
+// {count, rounds, total, n_r[64], a_r[64], tag} — tag written last
 size_t small_smem_bytes(u64 n, u64 E, u64 nwords);
 size_t small_smem_limit();
 size_t small_out_bytes();
 cudaError_t launch_small(cudaStream_t st, u32 n, u32 E, u32 nwords, const uint4* arcs, u32 s1,
-                         u32 pb, int* out, void* res);
+                         u32 pb, int* out, void* res, u64 tag);  // res: mapped host memory
 // max_ids: an upper bound of the forest size (n - 1) — sizes the staging of the id writes
 cudaError_t launch_output(cudaStream_t st, u32 nwords, const u32* msf, int* out, u32* tcnt,
                           u32* out_count, u32 max_ids);

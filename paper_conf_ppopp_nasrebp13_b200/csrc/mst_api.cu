@@ -158,6 +158,7 @@ struct mst_graph {
 
     bool opt_uf = false;     // MST_OPT_UNION_FIND (NEXT-3 variant)
     bool opt_small = true;   // MST_OPT_SMALL (one-CTA path for graphs that fit shared memory)
+    bool adj_dedup = true;   // A8's adjacent-duplicate filter in compacting passes (layout rule)
     bool opt_dedup = false;  // MST_OPT_DEDUP (A9: sort-based duplicate collapse after compaction)
     void* dd_scratch = nullptr;  // its scratch (allocated when the option is set)
     size_t dd_bytes = 0;
@@ -224,7 +225,7 @@ void release(mst_graph* g) {
     if (g->hacc) cudaFreeHost(g->hacc);
     if (g->hmap) cudaFreeHost((void*)g->hmap);
     if (g->xhost) cudaFreeHost(g->xhost);
-    if (g->small_host) cudaFreeHost(g->small_host);
+    if (g->small_host) cudaFreeHost(g->small_host);  // (mapped: small_res aliases it)
     if (g->trace) cudaFree(g->trace);
     for (auto e : g->evpool) cudaEventDestroy(e);
     if (g->fail_ev) cudaEventDestroy(g->fail_ev);
@@ -369,7 +370,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CK(cudaMemsetAsync(cursor, 0, std::max<u64>(n, 1) * sizeof(u32), g->cst));
     const char* ro = getenv("MST_REORDER");  // "0": the caller's numbering, "1": hub-first, "2": BFS
     std::vector<u32> hd;
-    bool bfs = ro && ro[0] == '2';
+    bool bfs = ro && ro[0] == '2' && nranks == 1;
     if (n > 0 && reorder && !ro) {
         // auto layout (NEXT-4, measured in DESIGN.md §5d): heavy-tailed degrees -> hub-first;
         // near-regular degrees whose ids carry no locality (mean |u - v| > n / 8: uniform,
@@ -380,9 +381,17 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
         CK(cudaStreamSynchronize(g->cst));
         const u32 dmax = *std::max_element(hd.begin(), hd.end());
         const bool heavy = (double)dmax * (double)n >= 16.0 * 2.0 * (double)m;
-        bfs = !heavy && m > 0 && (double)span / (double)m > (double)n / 8.0;
+        // (not for a distributed handle: the BFS order depends on atomics, and every rank
+        // must derive the identical numbering)
+        bfs = !heavy && m > 0 && (double)span / (double)m > (double)n / 8.0 && nranks == 1;
     }
     g->st.layout = (n > 0 && reorder && !(ro && ro[0] == '0')) ? (bfs ? 2 : 1) : 0;
+    // A8's adjacent-duplicate filter pays where parallel records sit next to each other (road:
+    // 2.50 -> 2.19 ms) and costs a little where the ids carry no locality (uniform +2 %)
+    {
+        static const char* ad = getenv("MST_ADJ_DEDUP");  // "0" / "1": force
+        g->adj_dedup = ad ? ad[0] == '1' : !bfs;
+    }
     if (n > 0 && reorder && bfs) {
         // NEXT-4 locality layout: BFS order from the highest-degree vertex (§6.1)
         if (hd.empty()) {
@@ -490,8 +499,11 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     // defers components (no merge) and switches to all edges before 3n + 1 is reached
     CKS(galloc(g, &g->maps, 3 * n + 1));
     CKS(galloc(g, &g->msf, g->nwords));
-    CKS(galloc(g, reinterpret_cast<unsigned char**>(&g->small_res), small_out_bytes()));
-    CK(cudaMallocHost(&g->small_host, small_out_bytes()));
+    // the one-CTA path's result block lives in mapped pinned memory: the kernel writes it and
+    // publishes a tag; the host spins on the tag (no copy, no stream synchronisation)
+    CK(cudaHostAlloc(&g->small_host, small_out_bytes(), cudaHostAllocMapped));
+    memset(g->small_host, 0, small_out_bytes());
+    CK(cudaHostGetDevicePointer(&g->small_res, g->small_host, 0));
     CKS(galloc(g, &g->phi, n));
     if (n >= 2) {  // dense min-matrices (A9 / NEXT-1), <= 67 MB each
         CKS(galloc(g, &g->mat[0], dense_entries(n)));
@@ -673,19 +685,29 @@ struct SmallHost {  // (the layout of kernels.cu SmallOut)
     u32 count, rounds;
     u64 total;
     u32 n_r[64], a_r[64];
+    u64 tag;
 };
 mst_status run_small(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out_num,
                      uint64_t* out_total, unsigned long long kl0) {
-    static_assert(sizeof(SmallHost) == 8 + 8 + 512, "SmallOut layout");
+    static_assert(sizeof(SmallHost) == 8 + 8 + 512 + 8, "SmallOut layout");
     const u64 n = g->n, E = g->shards[0].hi - g->shards[0].lo;
+    const u64 tag = ((u64)(++g->run_seq) << 1) | 1u;  // (never 0: the initial value)
     {
         Prof p(g, s, MST_K_SMALL, 0);
         CK(launch_small(s, (u32)n, (u32)E, (u32)g->nwords, g->arcs0 + g->shards[0].lo,
-                        g->kfmt & 0xffu, g->kfmt >> 8, out_ids, g->small_res));
+                        g->kfmt & 0xffu, g->kfmt >> 8, out_ids, g->small_res, tag));
     }
-    CK(cudaMemcpyAsync(g->small_host, g->small_res, sizeof(SmallHost), cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
-    const SmallHost* h = reinterpret_cast<const SmallHost*>(g->small_host);
+    volatile SmallHost* vh = reinterpret_cast<volatile SmallHost*>(g->small_host);
+    for (u64 spin = 0; vh->tag != tag; ++spin) {  // (the stream is checked now and then)
+        if ((spin & 4095) == 4095) {
+            const cudaError_t e = cudaStreamQuery(s);
+            if (e != cudaSuccess && e != cudaErrorNotReady)
+                return fail(MST_ECUDA, "one-CTA path: %s", cudaGetErrorString(e));
+            if (e == cudaSuccess && vh->tag != tag) return fail(MST_EINTERNAL, "one-CTA path: no result");
+        }
+    }
+    if (g->prof) CK(cudaStreamSynchronize(s));  // (the profiling events)
+    const SmallHost* h = const_cast<const SmallHost*>(reinterpret_cast<volatile SmallHost*>(g->small_host));
     g->st.rounds = (int32_t)std::min<u32>(h->rounds, MST_MAX_ROUNDS);
     for (int r = 0; r < g->st.rounds; ++r) {
         g->st.n_r[r] = h->n_r[r];
@@ -769,7 +791,7 @@ mst_status run_uf(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out_n
             CK(launch_uf_pass(s, g->nsm, g->dcnt + arec(0, r), sh.hi - sh.lo, cur, parent,
                               never ? nullptr : const_cast<uint4*>(outbuf), g->bestA, (u32)n,
                               g->status, g->epoch++, g->dcnt + arec(0, r + 1), g->dcnt + C_TILE,
-                              g->pass_seq, cc, g->kfmt, tag));
+                              g->pass_seq, cc, g->kfmt, tag, g->adj_dedup));
         }
         {
             Prof p(g, s, MST_K_HOOK, r);
@@ -1325,7 +1347,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                                      to_dense ? g->mat[0] : nullptr, ccj,
                                      (to_dense && use_hub_row(g) && hub_ok)
                                          ? (const int*)g->dcnt + C_HUB + r + 1 : nullptr,
-                                     g->kfmt));
+                                     g->kfmt, g->adj_dedup));
             }
             if (to_dense && use_hub_row(g) && hub_ok) g->st.hub_row = 1;
             if (member) {

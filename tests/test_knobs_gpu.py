@@ -40,6 +40,9 @@ KNOBS = [
     {"MST_LIGHT_ONLY0": "1"},
     {"MST_LIGHT_ONLY0": "0"},
     {"MST_MEMBER_SCAN": "0"},    # always a pass over every record after the light phase
+    {"MST_ADJ_DEDUP": "0"},      # no adjacent-duplicate filter in compacting passes
+    {"MST_ADJ_DEDUP": "1"},      # ... on everywhere (also BFS-ordered graphs)
+    {"MST_REORDER": "1"},        # hub-first even where the auto rule picks BFS order
     {"MST_SMALL": "0"},          # no one-CTA path (grid64 through the multi-kernel path)
     {"MST_TEST_OPTIONS": "6=1"},                     # union-find variant (NEXT-3)
     {"MST_TEST_OPTIONS": "6=1", "MST_UF_TAG": "0"},  # ... untagged keys, best reset per round

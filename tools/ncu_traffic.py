@@ -25,13 +25,16 @@ for r in rows[2:]:
     b = sum(float(r[i[k]]) * scale[units[i[k]]] for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"))
     launches.append({"kernel": name.split("(")[0], "dram_bytes": b,
                      "us": float(r[i["gpu__time_duration.sum"]])})
-filt = [x for x in launches if "k_arc_pass<1" in x["kernel"]]
-min0 = [x for x in launches if "k_arc_pass<0" in x["kernel"]]
+filt = [x for x in launches if "k_arc_pass<1" in x["kernel"] or "k_arc_pass<(int)1" in x["kernel"]
+        or "k_member_min" in x["kernel"]]
+min0 = [x for x in launches if "k_arc_pass<0" in x["kernel"] or "k_arc_pass<(int)0" in x["kernel"]]
+small = [x for x in launches if "k_small_msf" in x["kernel"]]
 res = {"workload": wl, "kernel": "k_arc_pass<MODE_FILTER> (A8) / <MODE_MIN0> (A2)",
        "source": f"ncu --set full --clock-control none ({cmd})",
        "launches": launches,
        "per_launch_dram_bytes": [x["dram_bytes"] for x in filt],
        "filter_dram_bytes_per_launch": sum(x["dram_bytes"] for x in filt) / max(len(filt), 1),
-       "min0_dram_bytes_per_launch": sum(x["dram_bytes"] for x in min0) / max(len(min0), 1)}
+       "min0_dram_bytes_per_launch": sum(x["dram_bytes"] for x in min0) / max(len(min0), 1),
+       "small_dram_bytes_per_launch": sum(x["dram_bytes"] for x in small) / max(len(small), 1)}
 json.dump(res, open(f"profiles/ncu_traffic_{wl}.json", "w"), indent=1)
 print(json.dumps(res, indent=1))

@@ -5,7 +5,7 @@ WL=${WL:-rmat22}
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_$WL.csv \
     python bench.py --workload $WL --steps 2 --warmup 3 --e2e-steps 0 --no-oracle > /dev/null 2>&1
 # the bench runs warmup + 2 x steps mst_run calls: capture the arc passes of the LAST run only
-RE=${RE:-arc_pass}
+RE=${RE:-arc_pass|k_member_min|k_small_msf}
 SKIP=$(python - "$WL" "$RE" <<'PY'
 import csv, re, sys
 wl, rx = sys.argv[1], re.compile(sys.argv[2])
