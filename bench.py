@@ -141,7 +141,7 @@ def byte_model(st):
         dense = dr >= 0 and r >= dr
         if r == R - 1:
             out.append({"kind": "hook-only", "bytes": 0})
-        elif me[r] >= 0:  # member-scan round: the record ends it read (16 B each)
+        elif me[r] >= 0 and r > 0:  # member-scan round: the record ends it read (16 B each)
             out.append({"kind": "member", "compacted": False, "bytes": 16 * me[r]})
         elif dense:
             out.append({"kind": "dense", "bytes": 8 * a[r]})
@@ -170,6 +170,8 @@ def launch_bytes(st, lt, bm):
     light = st.get("light_t", 0xFFFFFFFF) != 0xFFFFFFFF
     if lt["kind"] == "min0":
         wrote = 16 * st["a_r"][0] if light and st["rounds"] else 0
+        if lt["sub"] == "singletons":  # the record ends it read (member_ends[0])
+            return 16 * max(st.get("member_ends", [0])[0], 0)
         return 16 * st["local_arcs0"] + wrote if lt["sub"] in ("min_all", "extract") else wrote
     if lt["kind"] == "filter" and lt["round"] < len(bm):
         return bm[lt["round"]]["bytes"]

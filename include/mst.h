@@ -136,7 +136,8 @@ enum {
 /* launch sub-kinds (mst_launch_time.sub), so unlike launches of one kind are told apart:
  *   MST_K_MIN0  : MIN_ALL   = minima over every record (+ the light-record write);
  *                 EXTRACT   = light-only round 0: the light-record write alone;
- *                 MIN_LIGHT = minima over the light records
+ *                 MIN_LIGHT = minima over the light records; SINGLETONS = the minima of
+ *                 the vertices without a light record, from their own records
  *   MST_K_FILTER: SPARSE = a pass over the alive records; LIGHT = a light-edge phase pass;
  *                 SWITCH = the pass that re-reads every record after the light phase;
  *                 TRANSITION = the pass into the dense min-matrix; MEMBER = a member-scan round
@@ -144,7 +145,7 @@ enum {
  *                 records, after the light-edge phase)
  *   MST_K_DENSE : DENSE_ROUND, DENSE_BEST, TAIL (the cooperative device tail) */
 enum {
-    MST_SUB_MIN_ALL = 0, MST_SUB_EXTRACT = 1, MST_SUB_MIN_LIGHT = 2,
+    MST_SUB_MIN_ALL = 0, MST_SUB_EXTRACT = 1, MST_SUB_MIN_LIGHT = 2, MST_SUB_SINGLETONS = 3,
     MST_SUB_SPARSE = 0, MST_SUB_LIGHT = 1, MST_SUB_SWITCH = 2, MST_SUB_TRANSITION = 3,
     MST_SUB_MEMBER = 4,
     MST_SUB_DENSE_ROUND = 0, MST_SUB_DENSE_BEST = 1, MST_SUB_TAIL = 2
@@ -178,7 +179,8 @@ typedef struct {
     uint32_t light_t;                     /* its weight threshold (light: w <= light_t);
                                              0xffffffff when the phase was off            */
     int64_t member_ends[MST_MAX_ROUNDS];  /* member-scan round r: record ends read (the
-                                             members' own + reverse records); -1: not one */
+                                             members' own + reverse records); -1: not one;
+                                             [0]: round 0's singleton scan, if it ran     */
     int64_t dedup_in[MST_MAX_ROUNDS];     /* A9: records entering the dedup after round r's
                                              pass (a_r[r + 1] = after it); -1: none        */
     int32_t layout;                       /* internal vertex numbering of the build: 0 the

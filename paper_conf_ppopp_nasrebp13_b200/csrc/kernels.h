@@ -122,6 +122,11 @@ cudaError_t launch_member_work(cudaStream_t st, int nsm, u32 n, const int* phi, 
 cudaError_t launch_member_min(cudaStream_t st, int nsm, u32 n, const int* phi, const u32* row,
                               const u32* rrow, const u32* ridx, const uint4* arcs, u32 vlo,
                               u32 vhi, u32 wbase, u64* best, u32 kfmt);
+// round 0 after a light-only round-0 pass: best[v] = min over all of v's records for every v
+// whose best is still inf (no light record); *ends += record ends read
+cudaError_t launch_singleton_min(cudaStream_t st, int nsm, u32 n, u64* best, const u32* row,
+                                 const u32* rrow, const u32* ridx, const uint4* arcs, u32 vlo,
+                                 u32 vhi, u32 wbase, u32 kfmt, u64* ends);
 // the reverse index of the A local records (other endpoint -> record indices); rdeg, cursor:
 // n-word scratch; rrow: n + 1 words; ridx: A words
 cudaError_t launch_reverse_index(cudaStream_t st, int nsm, u32 n, u64 A, const uint4* arcs,

@@ -140,6 +140,7 @@ struct mst_graph {
     u64* dmap = nullptr;           // its device alias
     u32 run_seq = 0;
     u64* hacc = nullptr;  // pinned
+    u64* hscr = nullptr;  // pinned scratch: [0] member-scan work, [1] round 0's singleton ends
     int* out_tmp = nullptr;  // for mst_run_host
 
     std::vector<Shard> shards;  // local shards (1, or G in the simulation)
@@ -223,6 +224,7 @@ void release(mst_graph* g) {
     }
     if (g->hcnt) cudaFreeHost(g->hcnt);
     if (g->hacc) cudaFreeHost(g->hacc);
+    if (g->hscr) cudaFreeHost(g->hscr);
     if (g->hmap) cudaFreeHost((void*)g->hmap);
     if (g->xhost) cudaFreeHost(g->xhost);
     if (g->small_host) cudaFreeHost(g->small_host);  // (mapped: small_res aliases it)
@@ -333,6 +335,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CK(cudaMemsetAsync(g->dcnt, 0, DCNT_WORDS * sizeof(u32), g->cst));
     CK(cudaMallocHost(&g->hcnt, DCNT_WORDS * sizeof(u32)));
     CK(cudaMallocHost(&g->hacc, 2 * ACC_SLOTS * sizeof(u64)));
+    CK(cudaMallocHost(&g->hscr, 4 * sizeof(u64)));
     {
         void* hm = nullptr;
         CK(cudaHostAlloc(&hm, 2 * HSURV * sizeof(u64), cudaHostAllocMapped));
@@ -905,19 +908,23 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     // the light records (no minima over the full stream); the round-0 minima come from the
     // light records and vertices without one are deferred. K = 8 makes that a ~e^-16 event
     // per vertex on near-regular graphs (light degree ~ Poisson(2K)); it stays exact anyway.
+    // (with the reverse index, >= 8 records per vertex, round 0 stays exact for the vertices
+    // without a light record: their minima come from their own records, k_singleton_min, so
+    // the round-0 pass is a pure extraction there too — RMAT-22: 357 -> ~200 us)
     static const char* lo_env = getenv("MST_LIGHT_ONLY0");
+    static const char* me_env = getenv("MST_MEMBER_SCAN");  // "0": never (ablation)
+    const bool member_ok = g->ridx && !(me_env && me_env[0] == '0');
     const bool dense_regime = g->A0 >= 64ull * (u64)n;
-    const bool lo0_want = lo_env ? lo_env[0] == '1' : (g->light_k < 0 && dense_regime);
+    const bool lo0_want = lo_env ? lo_env[0] == '1' : (g->light_k < 0 && (dense_regime || member_ok));
     const u32 lk = lk_env != 0xffffffffu ? lk_env
-                 : g->light_k >= 0 ? (u32)g->light_k : (lo0_want ? 8u : 2u);
+                 : g->light_k >= 0 ? (u32)g->light_k : (dense_regime ? 8u : 2u);
     // (decided on the global record count E_0: every rank of a distributed run agrees)
     int phase = (lk > 0 && !g->opt_keep && g->A0 >= 4096 &&
                  g->A0 >= 4ull * lk * n) ? 1 : 0;  // light records <= a quarter
     const bool dist = g->xkind != X_NONE;
     const bool light_only0 = lo0_want && phase;
-    // member-scan rounds can finish the light phase (reverse index built: >= 8 records/vertex)
-    static const char* me_env = getenv("MST_MEMBER_SCAN");  // "0": never (ablation)
-    const bool member_ok = g->ridx && !(me_env && me_env[0] == '0');
+    // round-0 minima of the vertices without a light record from their own records
+    const bool singletons = light_only0 && member_ok;
     g->st.light_switch_round = -1;
     g->st.light_t = 0xffffffffu;
     if (phase) {
@@ -936,7 +943,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             // phase leaves are finished by member scans, not by a pass over every record;
             // measured on RMAT-22: t 139 -> 60, 62.8 -> 66.1 G edges/s; t 40: 64.9)
             const bool auto_k = lk_env == 0xffffffffu && g->light_k < 0;
-            const u64 target = !auto_k ? (u64)lk * n : lo0_want ? (u64)10 * n
+            const u64 target = !auto_k ? (u64)lk * n : dense_regime ? (u64)10 * n
                              : member_ok ? (u64)n : (u64)23 * n / 10;
             // a rank samples its own records, aimed at the same fraction of them; every rank
             // must use the SAME t (a mixed threshold is not a prefix of the (w, id) order),
@@ -985,7 +992,18 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     if (g->sim) {
         Prof p(g, s, MST_K_COMM, 0);
         CK(launch_combine_min(s, g->nsm, (u32)n, G, g->shard_best, n, g->bestA));
-    } else if (dist) {
+    }
+    if (singletons) {
+        // (a rank scans its own records for the vertices without a LOCAL light key: a vertex
+        // with a light record elsewhere keeps it through the MIN, light keys < heavy keys)
+        Prof p(g, s, MST_K_MIN0, 0, MST_SUB_SINGLETONS);
+        CK(cudaMemsetAsync(g->mwork, 0, sizeof(u64), s));
+        CK(launch_singleton_min(s, g->nsm, (u32)n, g->bestA, g->row, g->rrow, g->ridx, g->arcs0,
+                                g->vlo, g->vhi, g->wbase, g->kfmt, g->mwork));
+        // (stream-ordered before the member scans reuse the counter; read at the run's end)
+        CK(cudaMemcpyAsync(&g->hscr[1], g->mwork, sizeof(u64), cudaMemcpyDeviceToHost, s));
+    }
+    if (dist) {
         // edge-once records: a vertex's round-0 minimum has contributions from every rank
         // that owns one of its edges (the other endpoint's side), so round 0 needs a
         // reduction too, not an allgather of rank-local minima
@@ -1051,10 +1069,9 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                                   g->mwork));
         }
         ready = true;
-        CK(cudaMemcpyAsync(&g->hacc[2 * ACC_SLOTS - 1], g->mwork, sizeof(u64),
-                           cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(&g->hscr[0], g->mwork, sizeof(u64), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
-        work = g->hacc[2 * ACC_SLOTS - 1];
+        work = g->hscr[0];
         if (dist) {  // MAX over ranks = ~MIN(~x)
             u64 nx = ~work;
             CK(cudaMemcpyAsync(g->mwork, &nx, sizeof(u64), cudaMemcpyHostToDevice, s));
@@ -1143,7 +1160,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             Prof p(g, s, MST_K_HOOK, r);
             CK(launch_hook(s, nr, bcur, bnxt, g->dmap + r, tag_base | (u32)r, g->euv, chain, g->P,
                            g->Mtmp, g->msf, g->acc, g->tcnt, g->dcnt + C_NNEXT,
-                           phase == 1 && (r > 0 || light_only0),  // (else round 0's
+                           phase == 1 && (r > 0 || (light_only0 && !singletons)),  // (else round 0's
                                                                   // minima cover every edge)
                            dense ? 0u : g->kfmt));  // dense rounds: matrix keys (w << 32 | eid)
         }
@@ -1430,6 +1447,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         CKS(wait_word(g, s, HSURV + pend, tag_base | (u32)pend, &word));
         resolve(word);
     }
+    if (singletons) g->st.member_ends[0] = (int64_t)g->hscr[1];
     for (int i = 1; i < ACC_SLOTS; ++i) {  // sum the spread accumulators
         g->hacc[0] += g->hacc[2 * i];
         g->hacc[1] += g->hacc[2 * i + 1];

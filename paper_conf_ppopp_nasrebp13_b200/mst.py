@@ -23,7 +23,7 @@ K_INIT, K_MIN0, K_HOOK, K_JUMP, K_FILTER, K_OUTPUT, K_COMM, K_DENSE, K_LIGHT, K_
 KERNEL_NAMES = ["init", "min0", "hook", "jump", "filter", "output", "comm", "dense", "light",
                 "compose", "small", "dedup"]
 # launch sub-kinds per kind (include/mst.h MST_SUB_*)
-SUB_NAMES = {K_MIN0: ["min_all", "extract", "min_light"],
+SUB_NAMES = {K_MIN0: ["min_all", "extract", "min_light", "singletons"],
              K_FILTER: ["sparse", "light", "switch", "transition", "member"],
              K_DENSE: ["dense_round", "dense_best", "tail"],
              K_COMPOSE: ["compose", "sample"]}
