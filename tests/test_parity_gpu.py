@@ -3,6 +3,10 @@
 Compared on the same seeded inputs (graphgen): the ascending forest ids, their count and
 the exact uint64 total weight (integer work -> bit-exact, no tolerance).
 """
+import os
+import subprocess
+import sys
+
 import numpy as np
 import pytest
 
@@ -440,6 +444,38 @@ def test_light_only_round0_deferred(lib, oracle_mod):
     src = np.concatenate([s1, sp]).astype(np.int32)
     dst = np.concatenate([d1, dp]).astype(np.int32)
     w = np.concatenate([w1, wp]).astype(np.uint32)
+    st = assert_parity(lib, oracle_mod, n, src, dst, w, runs=2)
+    # the pendants got their exact round-0 minimum from their own records (the reverse index
+    # exists at >= 8 records per vertex: member_ends[0] = the record ends that scan read), or
+    # their edge after the switch to all records
+    assert st["light_t"] < 900
+    assert st["light_switch_round"] >= 0 or st["member_ends"][0] > 0
+    # without the member scans: deferred from round 0 on, the switch re-reads every record
+    env = dict(os.environ, MST_MEMBER_SCAN="0")
+    code = ("import sys; sys.path.insert(0, 'tests'); import numpy as np, test_parity_gpu as t, "
+            "paper_conf_ppopp_nasrebp13_b200 as p, oracle as o; p.load(); o.build(); "
+            "t.check_light_only_round0_no_member(p, o)")
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
+                       timeout=600, cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    assert r.returncode == 0, r.stderr[-3000:]
+
+
+def _light_only_graph():
+    rng = np.random.default_rng(11)
+    nc, npend, niso = 3000, 500, 50
+    n = nc + npend + niso
+    mc_ = 100 * nc
+    s1 = rng.integers(0, nc, mc_); d1 = rng.integers(0, nc, mc_); w1 = rng.integers(0, 100, mc_)
+    sp = np.repeat(np.arange(nc, nc + npend), 2); dp = rng.integers(0, nc, 2 * npend)
+    wp = rng.integers(900, 1000, 2 * npend)
+    src = np.concatenate([s1, sp]).astype(np.int32)
+    dst = np.concatenate([d1, dp]).astype(np.int32)
+    w = np.concatenate([w1, wp]).astype(np.uint32)
+    return n, src, dst, w
+
+
+def check_light_only_round0_no_member(lib, oracle_mod):
+    n, src, dst, w = _light_only_graph()
     st = assert_parity(lib, oracle_mod, n, src, dst, w, runs=2)
     assert st["light_t"] < 900 and st["light_switch_round"] >= 0
 
