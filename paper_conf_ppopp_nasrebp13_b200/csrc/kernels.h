@@ -117,11 +117,13 @@ cudaError_t launch_uf_hook(cudaStream_t st, int nsm, u32 n, u32* parent, const u
 // the component of vertex 0 (phi: vertex -> component); member minima of those components
 // (own records [row[v] - wbase, row[v+1] - wbase) for owners in [vlo, vhi), reverse records
 // ridx[rrow[v] .. rrow[v+1])), best[phi[0]] = KEY_DEFER
+// (both work counters also list those vertices: list[0 .. *lcnt))
 cudaError_t launch_member_work(cudaStream_t st, int nsm, u32 n, const int* phi, const u32* row,
-                               const u32* rrow, u32 vlo, u32 vhi, u64* work);
-cudaError_t launch_member_min(cudaStream_t st, int nsm, u32 n, const int* phi, const u32* row,
-                              const u32* rrow, const u32* ridx, const uint4* arcs, u32 vlo,
-                              u32 vhi, u32 wbase, u64* best, u32 kfmt);
+                               const u32* rrow, u32 vlo, u32 vhi, u64* work, u32* list, u32* lcnt);
+// the member minima of the listed vertices (nmax: an upper bound of *lcnt, sizes the grid)
+cudaError_t launch_member_min(cudaStream_t st, int nsm, u32 nmax, const u32* list, const u32* lcnt,
+                              const int* phi, const u32* row, const u32* rrow, const u32* ridx,
+                              const uint4* arcs, u32 vlo, u32 vhi, u32 wbase, u64* best, u32 kfmt);
 // round 0 after a light-only round-0 pass: best[v] = min over all of v's records for every v
 // whose best is still inf (no light record); *ends += record ends read
 cudaError_t launch_singleton_min(cudaStream_t st, int nsm, u32 n, u64* best, const u32* row,
@@ -153,7 +155,7 @@ cudaError_t launch_compose(cudaStream_t st, int nsm, u32 nb, const int* src, con
 // the component *giant (the member-scan decision)
 cudaError_t launch_compose_work(cudaStream_t st, int nsm, u32 nb, const int* src, const int* Mr,
                                 int* phi, const int* giant, const u32* row, const u32* rrow,
-                                u32 vlo, u32 vhi, u64* work);
+                                u32 vlo, u32 vhi, u64* work, u32* list, u32* lcnt);
 cudaError_t launch_sample_survival(cudaStream_t st, const uint4* in, const u32* a_ptr, const int* M,
                                    u32* num, u32* den);
 // A10 latency regime: the whole method in one CTA (records, component arrays and forest bits

@@ -90,7 +90,8 @@ constexpr int C_WMAX = C_LT + 1;                   // largest weight (build)
 constexpr int C_TAILN = C_WMAX + 1;                // light-phase tail: labels after it
 constexpr u32 LBLK_MIN = 32, LBLK_MAX = 256;      // light write: records per warp reservation
 constexpr int C_UFU = C_TAILN + 1;                 // union-find variant: unions per round
-constexpr int DCNT_WORDS = C_UFU + MST_MAX_ROUNDS;
+constexpr int C_MLIST = C_UFU + MST_MAX_ROUNDS;    // member scan: listed vertices
+constexpr int DCNT_WORDS = C_MLIST + 1;
 constexpr int HSURV = MST_MAX_ROUNDS + 1;  // mapped words: [0, HSURV) sizes, [HSURV, 2 HSURV) decisions
 
 struct Shard {
@@ -941,10 +942,11 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             // vertices without a light edge and one more all-records pass — stays unlikely)
             // (with member-scan rounds, fewer light records pay: the components the light
             // phase leaves are finished by member scans, not by a pass over every record;
-            // measured on RMAT-22: t 139 -> 60, 62.8 -> 66.1 G edges/s; t 40: 64.9)
+            // measured on RMAT-22: t 139 -> 60, 62.8 -> 66.1 G edges/s; t 40: 64.9; with the
+            // light-only round 0: t 60 / 50 / 40 -> 69.2 / 70.8 / 69.1)
             const bool auto_k = lk_env == 0xffffffffu && g->light_k < 0;
             const u64 target = !auto_k ? (u64)lk * n : dense_regime ? (u64)10 * n
-                             : member_ok ? (u64)n : (u64)23 * n / 10;
+                             : member_ok ? (u64)n * 85 / 100 : (u64)23 * n / 10;
             // a rank samples its own records, aimed at the same fraction of them; every rank
             // must use the SAME t (a mixed threshold is not a prefix of the (w, id) order),
             // so the ranks agree on the smallest sampled t
@@ -1053,11 +1055,14 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     // component; the busiest rank's count decides for every rank
     auto member_work = [&](int rr, const int* Mrr, bool hubk, bool& ready, u64& work) -> mst_status {
         CK(cudaMemsetAsync(g->mwork, 0, sizeof(u64), s));
+        CK(cudaMemsetAsync(g->dcnt + C_MLIST, 0, sizeof(u32), s));
+        // (the list of the vertices outside the hub's component lives in P: free from the
+        // jump of this round to the hook of the next)
         if (!ready && hubk) {  // one pass: compose + count (the hub's label is tracked)
             Prof p(g, s, MST_K_COMPOSE, rr, 2);
             CK(launch_compose_work(s, g->nsm, (u32)n, rr >= 1 && chain.len ? (brnd == rr - 1 ? chain.m[chain.len - 1] : g->phi) : nullptr,
                                    Mrr, g->phi, (const int*)g->dcnt + C_HUB + rr + 1, g->row,
-                                   g->rrow, g->vlo, g->vhi, g->mwork));
+                                   g->rrow, g->vlo, g->vhi, g->mwork, g->P, g->dcnt + C_MLIST));
         } else {
             if (!ready) {
                 Prof p(g, s, MST_K_COMPOSE, rr);
@@ -1066,7 +1071,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             }
             Prof p(g, s, MST_K_COMPOSE, rr, 2);
             CK(launch_member_work(s, g->nsm, (u32)n, g->phi, g->row, g->rrow, g->vlo, g->vhi,
-                                  g->mwork));
+                                  g->mwork, g->P, g->dcnt + C_MLIST));
         }
         ready = true;
         CK(cudaMemcpyAsync(&g->hscr[0], g->mwork, sizeof(u64), cudaMemcpyDeviceToHost, s));
@@ -1334,8 +1339,10 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                 // the members' records of every component but the top hub's (deferred); the
                 // records themselves are untouched: the next full pass reads all of them
                 Prof p(g, s, MST_K_FILTER, r, MST_SUB_MEMBER);
-                CK(launch_member_min(s, g->nsm, (u32)n, g->phi, g->row, g->rrow, g->ridx, g->arcs0,
-                                     g->vlo, g->vhi, g->wbase, g->sim ? g->shard_best : bnxt, g->kfmt));
+                CK(launch_member_min(s, g->nsm, (u32)std::min<u64>(n, mwork + 1), g->P,
+                                     g->dcnt + C_MLIST, g->phi, g->row, g->rrow, g->ridx,
+                                     g->arcs0, g->vlo, g->vhi, g->wbase,
+                                     g->sim ? g->shard_best : bnxt, g->kfmt));
                 for (int j = 0; j < G; ++j) {
                     g->hcnt[arec(j, r + 1)] = (u32)(g->shards[j].hi - g->shards[j].lo);
                     CK(cudaMemcpyAsync(g->dcnt + arec(j, r + 1), g->hcnt + arec(j, r + 1),
