@@ -141,7 +141,8 @@ def byte_model(st):
         dense = dr >= 0 and r >= dr
         if r == R - 1:
             out.append({"kind": "hook-only", "bytes": 0})
-        elif me[r] >= 0 and r > 0:  # member-scan round: the record ends it read (16 B each)
+        elif me[r] >= 0 and r > 0 and st.get("member_round", [1] * R)[r] == 1:
+            # member-scan round: the record ends it read (16 B each); no pass
             out.append({"kind": "member", "compacted": False, "bytes": 16 * me[r]})
         elif dense:
             out.append({"kind": "dense", "bytes": 8 * a[r]})
@@ -173,6 +174,8 @@ def launch_bytes(st, lt, bm):
         if lt["sub"] == "singletons":  # the record ends it read (member_ends[0])
             return 16 * max(st.get("member_ends", [0])[0], 0)
         return 16 * st["local_arcs0"] + wrote if lt["sub"] in ("min_all", "extract") else wrote
+    if lt["kind"] == "filter" and lt["sub"] == "member":  # (pure or next to a light pass)
+        return 16 * max(st.get("member_ends", [0] * (lt["round"] + 1))[lt["round"]], 0)
     if lt["kind"] == "filter" and lt["round"] < len(bm):
         return bm[lt["round"]]["bytes"]
     return 0

@@ -185,6 +185,8 @@ typedef struct {
                                              pass (a_r[r + 1] = after it); -1: none        */
     int32_t layout;                       /* internal vertex numbering of the build: 0 the
                                              caller's, 1 hub-first, 2 BFS order (NEXT-4)   */
+    int32_t member_round[MST_MAX_ROUNDS]; /* 1: round r was a member-scan round, 2: a hybrid
+                                             round (light pass + member scan), 0: neither */
 } mst_stats;
 
 mst_status mst_get_stats(const mst_graph* g, mst_stats* out);

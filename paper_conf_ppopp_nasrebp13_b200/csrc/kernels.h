@@ -114,16 +114,16 @@ cudaError_t launch_uf_hook(cudaStream_t st, int nsm, u32 n, u32* parent, const u
                            bool tagged, u64 tag, const uint2* euv, u32* P, u32* msf, u64* acc,
                            u32* unions, const u32* surv, u64* hmap, u32 htag);
 // member-scan rounds (after the light-edge phase): *work += record ends of the vertices outside
-// the component of vertex 0 (phi: vertex -> component); member minima of those components
-// (own records [row[v] - wbase, row[v+1] - wbase) for owners in [vlo, vhi), reverse records
-// ridx[rrow[v] .. rrow[v+1])), best[phi[0]] = KEY_DEFER
-// (both work counters also list those vertices: list[0 .. *lcnt))
+// the component of vertex 0 (phi: vertex -> component)
 cudaError_t launch_member_work(cudaStream_t st, int nsm, u32 n, const int* phi, const u32* row,
-                               const u32* rrow, u32 vlo, u32 vhi, u64* work, u32* list, u32* lcnt);
-// the member minima of the listed vertices (nmax: an upper bound of *lcnt, sizes the grid)
-cudaError_t launch_member_min(cudaStream_t st, int nsm, u32 nmax, const u32* list, const u32* lcnt,
-                              const int* phi, const u32* row, const u32* rrow, const u32* ridx,
-                              const uint4* arcs, u32 vlo, u32 vhi, u32 wbase, u64* best, u32 kfmt);
+                               const u32* rrow, u32 vlo, u32 vhi, u64* work);
+// member minima of the components outside an exclusion set: own records [row[v] - wbase,
+// row[v+1] - wbase) for owners in [vlo, vhi), reverse records ridx[rrow[v] .. rrow[v+1]).
+// hubs == nullptr: a member-scan round, the set is {phi[0]} and best[phi[0]] = KEY_DEFER;
+// else a hybrid round next to a light pass: the set is hubs[0..31] (launch_compose_work's)
+cudaError_t launch_member_min(cudaStream_t st, int nsm, u32 n, const int* hubs, const int* phi,
+                              const u32* row, const u32* rrow, const u32* ridx, const uint4* arcs,
+                              u32 vlo, u32 vhi, u32 wbase, u64* best, u32 kfmt);
 // round 0 after a light-only round-0 pass: best[v] = min over all of v's records for every v
 // whose best is still inf (no light record); *ends += record ends read
 cudaError_t launch_singleton_min(cudaStream_t st, int nsm, u32 n, u64* best, const u32* row,
@@ -152,10 +152,16 @@ cudaError_t launch_dense_tail(cudaStream_t st, int nsm, u32 n0, u64* best0, u64*
                               int defer = 0, int* map_out = nullptr, u32* n_out = nullptr);
 cudaError_t launch_compose(cudaStream_t st, int nsm, u32 nb, const int* src, const int* Mr, int* phi);
 // the same over vertex ids, also summing into *work the record ends of the vertices outside
-// the component *giant (the member-scan decision)
+// the hub set's components (the member-scan decision); hubs: 33 ints written first (the
+// sorted labels of the components of vertices 0..31 after Mr, then their number of distinct
+// live labels)
+// the hub set alone, from vertex ids through chain and Mr; its distinct-label count also to the
+// tagged mapped word hword ((tag << 32) | count)
+cudaError_t launch_hub_chain(cudaStream_t st, u32 n, const MapChain& chain, const int* Mr,
+                             int* hubs, u64* hword, u32 tag);
 cudaError_t launch_compose_work(cudaStream_t st, int nsm, u32 nb, const int* src, const int* Mr,
-                                int* phi, const int* giant, const u32* row, const u32* rrow,
-                                u32 vlo, u32 vhi, u64* work, u32* list, u32* lcnt);
+                                int* phi, int* hubs, const u32* row, const u32* rrow,
+                                u32 vlo, u32 vhi, u64* work);
 cudaError_t launch_sample_survival(cudaStream_t st, const uint4* in, const u32* a_ptr, const int* M,
                                    u32* num, u32* den);
 // A10 latency regime: the whole method in one CTA (records, component arrays and forest bits

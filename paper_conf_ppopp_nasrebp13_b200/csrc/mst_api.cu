@@ -73,6 +73,8 @@ mst_status fail(mst_status s, const char* fmt, ...) {
 
 u32 bits_of(u64 x) { u32 b = 0; while (x) { ++b; x >>= 1; } return b; }
 
+constexpr int HUBS_N = 32;  // (kernels.cu HUBS: the hub set's size)
+
 // device-counter slots
 enum { C_ERR = 0, C_OUT = 1, C_NNEXT = 2, C_TILE = 3, C_AREC = 8 };  // C_TILE: 2 slots
 // C_AREC: per shard j and round r, the alive arcs entering round r (written by round r-1's
@@ -90,9 +92,9 @@ constexpr int C_WMAX = C_LT + 1;                   // largest weight (build)
 constexpr int C_TAILN = C_WMAX + 1;                // light-phase tail: labels after it
 constexpr u32 LBLK_MIN = 32, LBLK_MAX = 256;      // light write: records per warp reservation
 constexpr int C_UFU = C_TAILN + 1;                 // union-find variant: unions per round
-constexpr int C_MLIST = C_UFU + MST_MAX_ROUNDS;    // member scan: listed vertices
-constexpr int DCNT_WORDS = C_MLIST + 1;
-constexpr int HSURV = MST_MAX_ROUNDS + 1;  // mapped words: [0, HSURV) sizes, [HSURV, 2 HSURV) decisions
+constexpr int DCNT_WORDS = C_UFU + MST_MAX_ROUNDS;
+constexpr int HSURV = MST_MAX_ROUNDS + 1;  // mapped words: [0, HSURV) sizes, [HSURV, 2 HSURV) decisions,
+constexpr int HHUB = 2 * HSURV;            // [2 HSURV, 3 HSURV) the hub sets' component counts
 
 struct Shard {
     u64 lo, hi;  // record window [lo, hi) in the handle's arcs0 and in the ping-pong buffers
@@ -157,6 +159,7 @@ struct mst_graph {
     u32 vlo = 0, vhi = 0, wbase = 0;     // owners of this handle's records, their first record
     u32 *rrow = nullptr, *ridx = nullptr;  // reverse index (member-scan rounds): other -> records
     u64* mwork = nullptr;                // member-scan work estimate (device)
+    int* hubs = nullptr;                 // the hub set of a member decision (33 ints, device)
 
     bool opt_uf = false;     // MST_OPT_UNION_FIND (NEXT-3 variant)
     bool opt_small = true;   // MST_OPT_SMALL (one-CTA path for graphs that fit shared memory)
@@ -339,8 +342,8 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CK(cudaMallocHost(&g->hscr, 4 * sizeof(u64)));
     {
         void* hm = nullptr;
-        CK(cudaHostAlloc(&hm, 2 * HSURV * sizeof(u64), cudaHostAllocMapped));
-        memset(hm, 0, 2 * HSURV * sizeof(u64));
+        CK(cudaHostAlloc(&hm, 3 * HSURV * sizeof(u64), cudaHostAllocMapped));
+        memset(hm, 0, 3 * HSURV * sizeof(u64));
         g->hmap = (volatile u64*)hm;
         CK(cudaHostGetDevicePointer((void**)&g->dmap, hm, 0));
     }
@@ -478,6 +481,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
         CKS(galloc(g, &g->rrow, n + 1));
         CKS(galloc(g, &g->ridx, A_loc));
         CKS(galloc(g, &g->mwork, 1));
+        CKS(galloc(g, &g->hubs, 64));
         CK(launch_reverse_index(g->cst, g->nsm, (u32)n, A_loc, g->arcs0, rdeg, g->rrow, cursor,
                                 g->ridx, g->status, g->epoch++));
     }
@@ -875,6 +879,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         g->st.n_r[r] = g->st.a_r[r] = 0;
         g->st.round_filter_ms[r] = 0;
         g->st.member_ends[r] = -1;
+        g->st.member_round[r] = 0;
         g->st.dedup_in[r] = -1;
     }
     if (n == 0) {
@@ -1053,16 +1058,16 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     // member-scan rounds (after the light-edge phase, kernels.cu "member-scan"): Ψ = vertex ->
     // round r+1 label composed (if not yet) together with the record ends outside the top hub's
     // component; the busiest rank's count decides for every rank
-    auto member_work = [&](int rr, const int* Mrr, bool hubk, bool& ready, u64& work) -> mst_status {
+    // nbig: the distinct components among the top hubs' (1: only the giant is big)
+    auto member_work = [&](int rr, const int* Mrr, bool hubk, bool& ready, u64& work,
+                           u32& nbig) -> mst_status {
         CK(cudaMemsetAsync(g->mwork, 0, sizeof(u64), s));
-        CK(cudaMemsetAsync(g->dcnt + C_MLIST, 0, sizeof(u32), s));
-        // (the list of the vertices outside the hub's component lives in P: free from the
-        // jump of this round to the hook of the next)
         if (!ready && hubk) {  // one pass: compose + count (the hub's label is tracked)
             Prof p(g, s, MST_K_COMPOSE, rr, 2);
             CK(launch_compose_work(s, g->nsm, (u32)n, rr >= 1 && chain.len ? (brnd == rr - 1 ? chain.m[chain.len - 1] : g->phi) : nullptr,
-                                   Mrr, g->phi, (const int*)g->dcnt + C_HUB + rr + 1, g->row,
-                                   g->rrow, g->vlo, g->vhi, g->mwork, g->P, g->dcnt + C_MLIST));
+                                   Mrr, g->phi, g->hubs, g->row,
+                                   g->rrow, g->vlo, g->vhi, g->mwork));
+            CK(cudaMemcpyAsync(&g->hscr[2], g->hubs + HUBS_N, sizeof(int), cudaMemcpyDeviceToHost, s));
         } else {
             if (!ready) {
                 Prof p(g, s, MST_K_COMPOSE, rr);
@@ -1071,13 +1076,15 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             }
             Prof p(g, s, MST_K_COMPOSE, rr, 2);
             CK(launch_member_work(s, g->nsm, (u32)n, g->phi, g->row, g->rrow, g->vlo, g->vhi,
-                                  g->mwork, g->P, g->dcnt + C_MLIST));
+                                  g->mwork));
         }
+        const bool hubset = !ready && hubk;
         ready = true;
         CK(cudaMemcpyAsync(&g->hscr[0], g->mwork, sizeof(u64), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
         work = g->hscr[0];
-        if (dist) {  // MAX over ranks = ~MIN(~x)
+        nbig = hubset ? (u32)*reinterpret_cast<int*>(&g->hscr[2]) : 1u;
+        if (dist) {  // MAX over ranks = ~MIN(~x) (nbig is replicated: the labels are)
             u64 nx = ~work;
             CK(cudaMemcpyAsync(g->mwork, &nx, sizeof(u64), cudaMemcpyHostToDevice, s));
             CKS(xchg_min(g, s, g->mwork, 1, false));
@@ -1091,7 +1098,10 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     // worth it below ~1/16 of the streamed bytes)
     auto member_cheap = [&](u64 work) { return work * 16 < 2 * g->A0 / (u64)std::max(1, g->nranks); };
     bool member_next = false;  // the phase-1 check chose a member-scan round for this round
+    bool hybrid_next = false;  // ... a hybrid round: light pass + member scan of the small ones
+    bool hub_pending = false;  // the jump's hub set count is on its way to the host
     u64 member_w = 0;
+    u32 member_nbig = 1;
     bool dense = false;  // this round's alive arcs live in the min-matrix g->mat[mc]
     int mc = 0;
     g->st.dense_round = -1;
@@ -1157,6 +1167,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         int* Mr = g->maps + moff;
         u32 nn;
         const bool was_v = vround;
+        hub_pending = false;
         if (vround) {
             vround = false;
             nn = v_nn;
@@ -1175,6 +1186,12 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, g->tcnt, Mr, g->dcnt + C_NNEXT, bnxt,
                            (const int*)g->dcnt + C_HUB + r, (int*)g->dcnt + C_HUB + r + 1,
                            g->dmap + r, tag_base | (u32)r));
+        }
+        hub_pending = phase == 1 && member_ok && r >= 1 && !dense && brnd == 0 &&
+                      chain.len < MST_CHAIN_MAX;
+        if (hub_pending) {  // (the member-scan decision below first asks whether it can pay)
+            Prof p(g, s, MST_K_COMPOSE, r, 2);
+            CK(launch_hub_chain(s, (u32)n, chain, Mr, g->hubs, g->dmap + HHUB + r, tag_base | (u32)r));
         }
         // one host round trip per round: n_{r+1} (sizes round r's filter),
         // read zero-copy from the word the hook's last tile writes to mapped host memory
@@ -1198,16 +1215,27 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         static const char* sw_env = getenv("MST_LIGHT_SWITCH");
         const u64 sw_den = sw_env ? (u64)atoi(sw_env) : (member_ok ? (u64)n + 1 : 8);
         member_next = false;
-        if (phase == 1 && member_ok && r >= 1 && !was_v && !dense && hub_ok && brnd == 0 &&
-            nn > 1 && (u64)(nr - nn) * 2 < nr && moff + nr + 3ull * nn <= 3 * n) {
-            // light phase: once only the top hub's component is big (the others own few record
-            // ends), a member-scan round replaces both the next light pass and the pass over
-            // every record (RMAT-22: ~10 K small components, 2.37 M vertices in the giant)
-            CKS(member_work(r, Mr, true, phi_ready, member_w));
-            member_next = member_cheap(member_w);
+        hybrid_next = false;
+        static const char* hy_env = getenv("MST_HYBRID");
+        const bool hy = hy_env ? atoi(hy_env) != 0 : false;
+        u32 hub_comps = 0;
+        if (hub_pending && !was_v) CKS(wait_word(g, s, HHUB + r, tag_base | (u32)r, &hub_comps));
+        if (phase == 1 && member_ok && r >= 1 && !was_v && !dense && brnd == 0 && hub_pending &&
+            (hy || hub_comps <= 1) &&
+            nn > 1 && (u64)(nr - nn) * 4 < 3 * nr && moff + nr + 3ull * nn <= 3 * n) {
+            // light phase: once the components outside the top hubs' own few record ends, the
+            // member scan gives them their exact minima: next to a light pass while the hubs
+            // are still in several big pieces (a hybrid round: the pieces merge by their light
+            // minima), alone — replacing both the light pass and the pass over every record —
+            // once one giant is left (RMAT-22: ~10 K small components, 2.37 M vertices in it)
+            CKS(member_work(r, Mr, true, phi_ready, member_w, member_nbig));
+            const bool cheap = member_cheap(member_w);
+            member_next = cheap && member_nbig <= 1;
+            hybrid_next = hy && cheap && member_nbig > 1;
             static const bool dbg1 = getenv("MST_DEBUG_MEMBER") != nullptr;
-            if (dbg1) fprintf(stderr, "light round %d: nr %u nn %u member work %llu -> %d\n", r, nr,
-                              nn, (unsigned long long)member_w, (int)member_next);
+            if (dbg1) fprintf(stderr, "light round %d: nr %u nn %u member work %llu hub comps %u -> %d %d\n",
+                              r, nr, nn, (unsigned long long)member_w, member_nbig, (int)member_next,
+                              (int)hybrid_next);
         }
         if (phase == 1 && (member_next || was_v || nn == nr || (u64)(nr - nn) * sw_den < nr ||
                            moff + nr + 3ull * nn > 3 * n)) {
@@ -1253,7 +1281,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                 member = true;  // (decided by the phase-1 check of this round)
             } else if (phase == 2 && member_ok && cur == g->arcs0 && brnd == 0 &&
                        (phi_ready || brnd < r)) {
-                CKS(member_work(r, Mr, hub_ok, phi_ready, mwork));
+                u32 nbig = 1;
+                CKS(member_work(r, Mr, false, phi_ready, mwork, nbig));
                 member = member_cheap(mwork);
                 static const bool dbg = getenv("MST_DEBUG_MEMBER") != nullptr;
                 if (dbg) {
@@ -1335,12 +1364,20 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                     cc.den = g->dcnt + C_SEEN + (r - 1);
                 }
             }
+            if (hybrid_next && phase == 1 && !to_dense) {
+                // hybrid round: the small components' exact minima next to the light pass below
+                Prof p(g, s, MST_K_FILTER, r, MST_SUB_MEMBER);
+                CK(launch_member_min(s, g->nsm, (u32)n, g->hubs, g->phi, g->row, g->rrow, g->ridx,
+                                     g->arcs0, g->vlo, g->vhi, g->wbase,
+                                     g->sim ? g->shard_best : bnxt, g->kfmt));
+                g->st.member_ends[r] = (int64_t)member_w;
+                g->st.member_round[r] = 2;
+            }
             if (member) {
                 // the members' records of every component but the top hub's (deferred); the
                 // records themselves are untouched: the next full pass reads all of them
                 Prof p(g, s, MST_K_FILTER, r, MST_SUB_MEMBER);
-                CK(launch_member_min(s, g->nsm, (u32)std::min<u64>(n, mwork + 1), g->P,
-                                     g->dcnt + C_MLIST, g->phi, g->row, g->rrow, g->ridx,
+                CK(launch_member_min(s, g->nsm, (u32)n, nullptr, g->phi, g->row, g->rrow, g->ridx,
                                      g->arcs0, g->vlo, g->vhi, g->wbase,
                                      g->sim ? g->shard_best : bnxt, g->kfmt));
                 for (int j = 0; j < G; ++j) {
@@ -1349,6 +1386,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                                        sizeof(u32), cudaMemcpyHostToDevice, s));
                 }
                 g->st.member_ends[r] = (int64_t)mwork;
+                g->st.member_round[r] = 1;
             }
             for (int j = 0; j < G && !member; ++j) {
                 Shard& sh = g->shards[j];

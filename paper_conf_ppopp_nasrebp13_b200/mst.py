@@ -62,6 +62,7 @@ class mst_stats(ctypes.Structure):
         ("member_ends", ctypes.c_int64 * MAX_ROUNDS),
         ("dedup_in", ctypes.c_int64 * MAX_ROUNDS),
         ("layout", ctypes.c_int32),
+        ("member_round", ctypes.c_int32 * MAX_ROUNDS),
     ]
 
 
@@ -262,6 +263,7 @@ class MSTGraph:
             "member_ends": list(s.member_ends[:R]),
             "dedup_in": list(s.dedup_in[:R]),
             "layout": ["caller", "hub-first", "bfs"][s.layout] if 0 <= s.layout < 3 else s.layout,
+            "member_round": list(s.member_round[:R]),
         }
 
     def launch_times(self) -> list:
