@@ -12,6 +12,7 @@ for tool in ${TOOLS:-memcheck synccheck racecheck}; do
       echo "unique hazard locations (count, kernel, line):";
       grep -oE "at mstk::[a-zA-Z0-9_]+[^ ]* .*in [a-zA-Z0-9_.]+:[0-9]+" /tmp/san_$tool.log | \
         sed -E 's/\(.*\)\+0x[0-9a-f]+//' | sort | uniq -c | sort -rn | head -40; } > gpurun_out/sanitize_$tool.log
+    head -c 4000000 /tmp/san_$tool.log | gzip > gpurun_out/sanitize_${tool}_head.log.gz
   else
     cp /tmp/san_$tool.log gpurun_out/sanitize_$tool.log
   fi
