@@ -72,9 +72,10 @@ mst_status mst_create(int64_t n, int64_t m, const int32_t* src, const int32_t* d
                       const uint32_t* w, mst_graph** out);
 
 /* mst_create_host — as mst_create but src/dst/w are HOST pointers (pageable or pinned).
- * Pinned (page-locked) arrays are read by the build kernels directly over PCIe (zero-copy,
- * the transfer overlaps the validation and scatter passes); pageable arrays are first staged
- * through a device copy (input transferred to the GPU). */
+ * The arrays are copied to stream-ordered device buffers first (copy engines; pinned arrays
+ * reach the bus rate, ~55 GB/s, pageable ones are staged by the driver), then built as by
+ * mst_create (input transferred to the GPU). The build's small pinned host
+ * buffers come from a process-wide free list (no page-locking per handle). */
 mst_status mst_create_host(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                            const uint32_t* w, mst_graph** out);
 
@@ -100,9 +101,10 @@ mst_status mst_run_host(mst_graph* g, mst_stream_t stream, int32_t* out_edge_ids
 
 /* mst_solve_host — one end-to-end call from host arrays to host results:
  * mst_create_host + mst_run_host + mst_destroy. Device memory comes from a stream-ordered
- * pool that the library keeps between calls, so repeated solves do not pay cudaMalloc. Being
- * one-shot, it skips the build's hub-first relabelling pass (it costs more than one run
- * saves); the result is identical. */
+ * pool that the library keeps between calls, so repeated solves do not pay cudaMalloc. The
+ * build uses the automatic layout except the BFS order, and lays down no reverse index (the
+ * member-scan rounds' ~2 ms build pass, which one run does not repay; the BFS pass costs
+ * ~10 ms: those graphs keep the caller's numbering); the result is identical either way. */
 mst_status mst_solve_host(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                           const uint32_t* w, int32_t* out_edge_ids_host,
                           int64_t* out_num_edges, uint64_t* out_total_weight);

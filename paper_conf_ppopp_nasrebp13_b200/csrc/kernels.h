@@ -52,6 +52,8 @@ cudaError_t launch_reorder_bfs(cudaStream_t st, int nsm, u32 n, u32 m, const u32
                                u32* eu, u32* ev, u32* off, u32* cursor, u32* adj, u32* q,
                                u32* newid, u32* stt, u64* status, u32 epoch, u32* odeg,
                                int hi_owner, u32 root);
+// *out = max (deg[v] << 32 | ~v): the largest degree and the lowest vertex with it
+cudaError_t launch_deg_argmax(cudaStream_t st, int nsm, u32 n, const u32* deg, u64* out);
 cudaError_t launch_owner_degree(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
                                 u32* odeg, int hi_owner);
 cudaError_t launch_scatter(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
@@ -131,9 +133,10 @@ cudaError_t launch_singleton_min(cudaStream_t st, int nsm, u32 n, u64* best, con
                                  u32 vhi, u32 wbase, u32 kfmt, u64* ends);
 // the reverse index of the A local records (other endpoint -> record indices); rdeg, cursor:
 // n-word scratch; rrow: n + 1 words; ridx: A words
+u64 reverse_index_scratch(int nsm, u32 n);  // u32 words of launch_reverse_index's pc
 cudaError_t launch_reverse_index(cudaStream_t st, int nsm, u32 n, u64 A, const uint4* arcs,
                                  u32* rdeg, u32* rrow, u32* cursor, u32* ridx, u64* status,
-                                 u32 epoch);
+                                 u32 epoch, u32* pc);
 // A9 (MST_OPT_DEDUP, dedup.cu): sort the A records {s', d', key base} in rec (labels < nlab) by
 // their pair (min, max) and keep the minimum key of every pair, in place; *a_count = records
 // left (written on the device). scratch: dedup_scratch_bytes(A) bytes; nruns: one device int

@@ -23,6 +23,7 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <mutex>
 #include <new>
 #include <string>
 #include <vector>
@@ -137,6 +138,7 @@ struct mst_graph {
     u32 pass_seq = 0;  // TMA arc-pass launches (tile-counter slot parity)
     u32* dcnt = nullptr;
     u64* acc = nullptr;
+    void* hblock = nullptr;  // the pinned block (pinned_get) hcnt .. small_host live in
     u32* hcnt = nullptr;  // pinned
     volatile u64* hmap = nullptr;  // pinned + mapped: tagged n_{r+1} written by the hook,
                                    // then (at HSURV + r) the sampled compaction decision
@@ -193,6 +195,47 @@ struct mst_graph {
 
 namespace {
 
+// The handle's small pinned host buffers (counters, the mapped round words, the one-CTA result
+// block) live in one mapped block taken from a process-wide free list: pinning and unpinning
+// host memory costs milliseconds per handle (measured: 1.4-6 ms of a one-shot solve), and a
+// released block is zeroed and reused by the next handle.
+struct PinnedBlocks {
+    std::mutex mu;
+    std::vector<void*> free;
+};
+PinnedBlocks& pinned_blocks() {
+    static PinnedBlocks* p = new PinnedBlocks();  // (never destroyed: outlives every handle)
+    return *p;
+}
+void* pinned_get(size_t bytes) {
+    void* q = nullptr;
+    {
+        PinnedBlocks& pb = pinned_blocks();
+        std::lock_guard<std::mutex> lk(pb.mu);
+        if (!pb.free.empty()) {
+            q = pb.free.back();
+            pb.free.pop_back();
+        }
+    }
+    if (!q && cudaHostAlloc(&q, bytes, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) {
+        (void)cudaGetLastError();
+        return nullptr;
+    }
+    memset(q, 0, bytes);
+    return q;
+}
+void pinned_put(void* q) {
+    if (!q) return;
+    PinnedBlocks& pb = pinned_blocks();
+    std::lock_guard<std::mutex> lk(pb.mu);
+    pb.free.push_back(q);
+}
+constexpr size_t al64(size_t x) { return (x + 63) & ~(size_t)63; }
+size_t pinned_block_bytes() {  // hcnt | hacc | hscr | hmap | small_host
+    return al64(DCNT_WORDS * sizeof(u32)) + al64(2 * ACC_SLOTS * sizeof(u64)) +
+           al64(4 * sizeof(u64)) + al64(3 * HSURV * sizeof(u64)) + al64(small_out_bytes());
+}
+
 // keep freed pool memory reserved for the next handle (per device, idempotent, thread-safe)
 mst_status configure_pool(int dev) {
     cudaMemPool_t pool;
@@ -226,12 +269,8 @@ void release(mst_graph* g) {
         for (void* p : g->allocs) cudaFreeAsync(p, g->cst);
         cudaStreamSynchronize(g->cst);
     }
-    if (g->hcnt) cudaFreeHost(g->hcnt);
-    if (g->hacc) cudaFreeHost(g->hacc);
-    if (g->hscr) cudaFreeHost(g->hscr);
-    if (g->hmap) cudaFreeHost((void*)g->hmap);
+    pinned_put(g->hblock);  // (hcnt, hacc, hscr, hmap and small_host live in it)
     if (g->xhost) cudaFreeHost(g->xhost);
-    if (g->small_host) cudaFreeHost(g->small_host);  // (mapped: small_res aliases it)
     if (g->trace) cudaFree(g->trace);
     for (auto e : g->evpool) cudaEventDestroy(e);
     if (g->fail_ev) cudaEventDestroy(g->fail_ev);
@@ -319,9 +358,23 @@ mst_status shard_ranges(mst_graph* g, int G, std::vector<u64>& lo, std::vector<u
 }
 
 mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w, int nshards_sim,
-                 int rank, int nranks, bool reorder) {
+                 int rank, int nranks, int reorder) {
     auto t0 = std::chrono::steady_clock::now();
     const u64 n = g->n, m = g->m;
+    // reorder: 0 the caller's numbering, 1 the automatic layout, 2 a one-shot solve's (no BFS
+    // order, no reverse index: builds that one run does not repay)
+    const bool one_shot = reorder == 2;
+    // MST_TRACE_BUILD=1: the build's phases timed on the host (a stream sync at each mark)
+    static const bool btrace = getenv("MST_TRACE_BUILD") && getenv("MST_TRACE_BUILD")[0] == '1';
+    auto tmark = t0;
+    auto mark = [&](const char* what) {
+        if (!btrace) return;
+        cudaStreamSynchronize(g->cst);
+        const auto now = std::chrono::steady_clock::now();
+        fprintf(stderr, "build %-22s %8.3f ms\n", what,
+                std::chrono::duration<double, std::milli>(now - tmark).count());
+        tmark = now;
+    };
     g->nwords = (m + 31) / 32;
     CKS(galloc(g, &g->eu, m));
     CKS(galloc(g, &g->ev, m));
@@ -337,29 +390,38 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CK(cudaMemsetAsync(g->status, 0, nslots * sizeof(u64), g->cst));
     CK(cudaMemsetAsync(deg, 0, std::max<u64>(n, 1) * sizeof(u32), g->cst));
     CK(cudaMemsetAsync(g->dcnt, 0, DCNT_WORDS * sizeof(u32), g->cst));
-    CK(cudaMallocHost(&g->hcnt, DCNT_WORDS * sizeof(u32)));
-    CK(cudaMallocHost(&g->hacc, 2 * ACC_SLOTS * sizeof(u64)));
-    CK(cudaMallocHost(&g->hscr, 4 * sizeof(u64)));
     {
-        void* hm = nullptr;
-        CK(cudaHostAlloc(&hm, 3 * HSURV * sizeof(u64), cudaHostAllocMapped));
-        memset(hm, 0, 3 * HSURV * sizeof(u64));
-        g->hmap = (volatile u64*)hm;
-        CK(cudaHostGetDevicePointer((void**)&g->dmap, hm, 0));
+        char* hb = (char*)pinned_get(pinned_block_bytes());
+        if (!hb) return fail(MST_ENOMEM, "pinned host block of %zu bytes", pinned_block_bytes());
+        g->hblock = hb;
+        g->hcnt = (u32*)hb;
+        hb += al64(DCNT_WORDS * sizeof(u32));
+        g->hacc = (u64*)hb;
+        hb += al64(2 * ACC_SLOTS * sizeof(u64));
+        g->hscr = (u64*)hb;
+        hb += al64(4 * sizeof(u64));
+        g->hmap = (volatile u64*)hb;
+        CK(cudaHostGetDevicePointer((void**)&g->dmap, hb, 0));
+        hb += al64(3 * HSURV * sizeof(u64));
+        g->small_host = hb;
     }
 
-    u64* dspan;
-    CKS(galloc(g, &dspan, 1));
+    mark("allocations");
+    u64* dspan;  // [0] sum of |u - v|, [1] the degree argmax
+    CKS(galloc(g, &dspan, 2));
     CK(cudaMemsetAsync(dspan, 0, sizeof(u64), g->cst));
     CK(launch_degree(g->cst, g->nsm, (u32)n, (u32)m, src, dst, w, g->eu, g->ev, deg,
                      g->dcnt + C_ERR, g->dcnt + C_WMAX, dspan));
-    u64 span = 0;
+    CK(launch_deg_argmax(g->cst, g->nsm, (u32)n, deg, dspan + 1));
+    u64 span = 0, dtop = 0;
     CK(cudaMemcpyAsync(&span, dspan, sizeof(u64), cudaMemcpyDeviceToHost, g->cst));
+    CK(cudaMemcpyAsync(&dtop, dspan + 1, sizeof(u64), cudaMemcpyDeviceToHost, g->cst));
     CK(cudaMemcpyAsync(g->hcnt, g->dcnt, sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
     CK(cudaMemcpyAsync(g->hcnt + C_WMAX, g->dcnt + C_WMAX, sizeof(u32), cudaMemcpyDeviceToHost,
                        g->cst));
     CK(cudaStreamSynchronize(g->cst));
     if (g->hcnt[0]) return fail(MST_EINVAL, "an endpoint is outside [0, n) (n = %lld)", (long long)n);
+    mark("degree (reads inputs)");
     {   // packed minima keys when weight, edge id and a label fit in 63 bits (every handle:
         // the keys' order is the (w, eid) order, so the MIN of a distributed run is unchanged);
         // the records carry their key base, so the format is fixed before they are built
@@ -376,23 +438,24 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     const int hi_owner = (op && op[0] == '0') ? 0 : 1;
     CK(cudaMemsetAsync(cursor, 0, std::max<u64>(n, 1) * sizeof(u32), g->cst));
     const char* ro = getenv("MST_REORDER");  // "0": the caller's numbering, "1": hub-first, "2": BFS
-    std::vector<u32> hd;
+    const u32 dmax = (u32)(dtop >> 32), droot = ~(u32)dtop;  // (device argmax: no n-word copy)
     bool bfs = ro && ro[0] == '2' && nranks == 1;
     if (n > 0 && reorder && !ro) {
         // auto layout (NEXT-4, measured in DESIGN.md §5d): heavy-tailed degrees -> hub-first;
         // near-regular degrees whose ids carry no locality (mean |u - v| > n / 8: uniform,
         // dense) -> BFS order; near-regular with local ids (road, grids) -> hub-first, i.e.
         // the caller's order within equal degree buckets
-        hd.resize(n);
-        CK(cudaMemcpyAsync(hd.data(), deg, n * sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
-        CK(cudaStreamSynchronize(g->cst));
-        const u32 dmax = *std::max_element(hd.begin(), hd.end());
         const bool heavy = (double)dmax * (double)n >= 16.0 * 2.0 * (double)m;
         // (not for a distributed handle: the BFS order depends on atomics, and every rank
         // must derive the identical numbering)
         bfs = !heavy && m > 0 && (double)span / (double)m > (double)n / 8.0 && nranks == 1;
+        if (bfs && reorder == 2) {  // (a one-shot solve: the BFS build, ~10 ms, does not pay)
+            bfs = false;
+            reorder = 0;
+        }
     }
     g->st.layout = (n > 0 && reorder && !(ro && ro[0] == '0')) ? (bfs ? 2 : 1) : 0;
+    mark("layout decision");
     // A8's adjacent-duplicate filter pays where parallel records sit next to each other (road:
     // 2.50 -> 2.19 ms) and costs a little where the ids carry no locality (uniform +2 %)
     {
@@ -401,12 +464,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     }
     if (n > 0 && reorder && bfs) {
         // NEXT-4 locality layout: BFS order from the highest-degree vertex (§6.1)
-        if (hd.empty()) {
-            hd.resize(n);
-            CK(cudaMemcpyAsync(hd.data(), deg, n * sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
-            CK(cudaStreamSynchronize(g->cst));
-        }
-        const u32 root = (u32)(std::max_element(hd.begin(), hd.end()) - hd.begin());
+        const u32 root = droot;
         u32 *degn, *newid, *off, *bcur, *adj, *q, *stt;
         CKS(galloc(g, &degn, n));
         CKS(galloc(g, &newid, n));
@@ -439,6 +497,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     } else {
         CK(launch_owner_degree(g->cst, g->nsm, (u32)m, g->eu, g->ev, cursor, hi_owner));
     }
+    mark("renumbering");
     deg = cursor;
     u32* odeg_scan_out;
     CKS(galloc(g, &odeg_scan_out, n));
@@ -452,6 +511,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CK(cudaMemcpyAsync(&A0, g->row + n, sizeof(u32), cudaMemcpyDeviceToHost, g->cst));
     CK(cudaStreamSynchronize(g->cst));
     g->A0 = A0;  // every rank's records together (the global E_0: identical decisions)
+    mark("row offsets");
 
     // shards: owner-vertex ranges balanced by records. The simulation keeps
     // all G ranges in one handle; a distributed rank builds ONLY the records of its own range
@@ -473,7 +533,8 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     g->vlo = (u32)vlo;
     g->vhi = (u32)vhi;
     g->wbase = (u32)wbase;
-    if (n > 0 && (u64)A0 >= 8ull * n) {
+    mark("scatter (reads w)");
+    if (n > 0 && (u64)A0 >= 8ull * n && !one_shot) {
         // heavy-tailed / dense inputs (the light-edge phase's regime): the reverse index of the
         // records for the member-scan rounds (other endpoint -> record indices; build time only)
         u32* rdeg;
@@ -482,9 +543,12 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
         CKS(galloc(g, &g->ridx, A_loc));
         CKS(galloc(g, &g->mwork, 1));
         CKS(galloc(g, &g->hubs, 64));
+        u32* rpc;  // (per-CTA counts of the hot vertices; build time only)
+        CKS(galloc(g, &rpc, reverse_index_scratch(g->nsm, (u32)n)));
         CK(launch_reverse_index(g->cst, g->nsm, (u32)n, A_loc, g->arcs0, rdeg, g->rrow, cursor,
-                                g->ridx, g->status, g->epoch++));
+                                g->ridx, g->status, g->epoch++, rpc));
     }
+    mark("reverse index");
     g->shards.clear();
     // light-edge phase: each shard's light records and their dead filler records (at most
     // LBLK_MAX per consumer warp of the pass) get their own window in abuf[0]
@@ -509,15 +573,14 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CKS(galloc(g, &g->msf, g->nwords));
     // the one-CTA path's result block lives in mapped pinned memory: the kernel writes it and
     // publishes a tag; the host spins on the tag (no copy, no stream synchronisation)
-    CK(cudaHostAlloc(&g->small_host, small_out_bytes(), cudaHostAllocMapped));
-    memset(g->small_host, 0, small_out_bytes());
-    CK(cudaHostGetDevicePointer(&g->small_res, g->small_host, 0));
+    CK(cudaHostGetDevicePointer(&g->small_res, g->small_host, 0));  // (zeroed with the block)
     CKS(galloc(g, &g->phi, n));
     if (n >= 2) {  // dense min-matrices (A9 / NEXT-1), <= 67 MB each
         CKS(galloc(g, &g->mat[0], dense_entries(n)));
         CKS(galloc(g, &g->mat[1], dense_entries(n)));
     }
     CK(cudaStreamSynchronize(g->cst));
+    mark("rest");
     g->st.n = g->n;
     g->st.m = g->m;
     g->st.arcs0 = (int64_t)g->A0;
@@ -531,7 +594,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
 
 mst_status create_common(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                          const uint32_t* w, int nshards_sim, const uint8_t* id, int rank,
-                         int nranks, mst_graph** out, bool reorder = true,
+                         int nranks, mst_graph** out, int reorder = 1,
                          mst_allreduce_min_fn xfn = nullptr, void* xctx = nullptr) {
     if (!out) return fail(MST_EINVAL, "out is NULL");
     *out = nullptr;
@@ -1600,14 +1663,18 @@ static const void* device_alias(const void* p) {
 }
 
 static mst_status create_host_impl(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
-                                   const uint32_t* w, mst_graph** out, bool reorder) {
+                                   const uint32_t* w, mst_graph** out, int reorder) {
     if (!out) return fail(MST_EINVAL, "out is NULL");
     *out = nullptr;
     CKS(check_args(n, m, src, dst, w));
     int dev;
     CK(cudaGetDevice(&dev));
     CKS(configure_pool(dev));
-    if (m > 0) {
+    // (pinned host arrays are copied by DMA too: the build kernels reading them in place over
+    // the bus reached ~34 GB/s — measured 15.8 + 5.3 ms for RMAT-22's 805 MB — the copy
+    // engines ~55 GB/s)
+    static const char* zc = getenv("MST_HOST_ZEROCOPY");  // "1": read pinned inputs in place
+    if (m > 0 && zc && zc[0] == '1') {
         const void *as = device_alias(src), *ad = device_alias(dst), *aw = device_alias(w);
         if (as && ad && aw)
             return create_common(n, m, (const int32_t*)as, (const int32_t*)ad,
@@ -1641,7 +1708,7 @@ static mst_status create_host_impl(int64_t n, int64_t m, const int32_t* src, con
 
 mst_status mst_create_host(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                            const uint32_t* w, mst_graph** out) {
-    return guarded([&]() { return create_host_impl(n, m, src, dst, w, out, true); });
+    return guarded([&]() { return create_host_impl(n, m, src, dst, w, out, 1); });
 }
 
 mst_status mst_run(mst_graph* g, mst_stream_t stream, int32_t* out_edge_ids,
@@ -1687,8 +1754,11 @@ mst_status mst_solve_host(int64_t n, int64_t m, const int32_t* src, const int32_
                           const uint32_t* w, int32_t* out_ids_host, int64_t* out_num_edges,
                           uint64_t* out_total_weight) {
     mst_graph* g = nullptr;
-    // one-shot: no hub-first relabelling (its build pass costs more than one run saves)
-    mst_status s = guarded([&]() { return create_host_impl(n, m, src, dst, w, &g, false); });
+    // one-shot: the automatic layout too (hub-first costs ~1 ms of build and saves RMAT-22's
+    // member scans ~8 ms of run; MST_SOLVE_REORDER=0: the caller's numbering)
+    static const char* sr = getenv("MST_SOLVE_REORDER");
+    const int reorder = (sr && sr[0] == '0') ? 0 : 2;
+    mst_status s = guarded([&]() { return create_host_impl(n, m, src, dst, w, &g, reorder); });
     if (s != MST_OK) return s;
     s = mst_run_host(g, g->cst, out_ids_host, out_num_edges, out_total_weight);
     std::string keep = g_err;
