@@ -181,6 +181,7 @@ struct mst_graph {
     bool hub_row = false;
     u64* trace = nullptr;    // MST_TAIL_TRACE=1 (tools): phase timestamps of the dense tail    // heavy-tailed input: hub row of the dense transition in smem
     int* phi = nullptr;      // composed label map of the records' label space (row A7)
+    int* phi2 = nullptr;     // vertex -> component while phi maps compacted light records
 
     cudaEvent_t fail_ev = nullptr;  // recorded on the run stream when a run fails: the frees
                                     // of mst_destroy wait for whatever is still in flight
@@ -543,6 +544,7 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
         CKS(galloc(g, &g->ridx, A_loc));
         CKS(galloc(g, &g->mwork, 1));
         CKS(galloc(g, &g->hubs, 64));
+        CKS(galloc(g, &g->phi2, n));
         u32* rpc;  // (per-CTA counts of the hot vertices; build time only)
         CKS(galloc(g, &rpc, reverse_index_scratch(g->nsm, (u32)n)));
         CK(launch_reverse_index(g->cst, g->nsm, (u32)n, A_loc, g->arcs0, rdeg, g->rrow, cursor,
@@ -1122,27 +1124,37 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     // round r+1 label composed (if not yet) together with the record ends outside the top hub's
     // component; the busiest rank's count decides for every rank
     // nbig: the distinct components among the top hubs' (1: only the giant is big)
+    // (records still in vertex ids, brnd = 0: Ψ itself, ready for the pass too; compacted
+    // light records, brnd > 0: the spare map g->phi2 from the whole chain — it becomes Ψ only
+    // when the member round is taken, phi keeps the records' pass map otherwise)
     auto member_work = [&](int rr, const int* Mrr, bool hubk, bool& ready, u64& work,
                            u32& nbig) -> mst_status {
         CK(cudaMemsetAsync(g->mwork, 0, sizeof(u64), s));
+        const bool vs = brnd == 0;
+        int* vphi = vs ? g->phi : g->phi2;
+        const int* vsrc = rr >= 1 && chain.len ? (brnd == rr - 1 ? chain.m[chain.len - 1] : g->phi) : nullptr;
+        if (!vs) {
+            Prof p(g, s, MST_K_COMPOSE, rr);
+            CK(launch_chain_compose(s, g->nsm, (u32)n, chain, g->phi2));
+            vsrc = g->phi2;
+            ready = false;
+        }
         if (!ready && hubk) {  // one pass: compose + count (the hub's label is tracked)
             Prof p(g, s, MST_K_COMPOSE, rr, 2);
-            CK(launch_compose_work(s, g->nsm, (u32)n, rr >= 1 && chain.len ? (brnd == rr - 1 ? chain.m[chain.len - 1] : g->phi) : nullptr,
-                                   Mrr, g->phi, g->hubs, g->row,
+            CK(launch_compose_work(s, g->nsm, (u32)n, vsrc, Mrr, vphi, g->hubs, g->row,
                                    g->rrow, g->vlo, g->vhi, g->mwork));
             CK(cudaMemcpyAsync(&g->hscr[2], g->hubs + HUBS_N, sizeof(int), cudaMemcpyDeviceToHost, s));
         } else {
             if (!ready) {
                 Prof p(g, s, MST_K_COMPOSE, rr);
-                CK(launch_compose(s, g->nsm, (u32)n, brnd == rr - 1 ? chain.m[chain.len - 1] : g->phi,
-                                  Mrr, g->phi));
+                CK(launch_compose(s, g->nsm, (u32)n, vsrc, Mrr, vphi));
             }
             Prof p(g, s, MST_K_COMPOSE, rr, 2);
-            CK(launch_member_work(s, g->nsm, (u32)n, g->phi, g->row, g->rrow, g->vlo, g->vhi,
+            CK(launch_member_work(s, g->nsm, (u32)n, vphi, g->row, g->rrow, g->vlo, g->vhi,
                                   g->mwork));
         }
         const bool hubset = !ready && hubk;
-        ready = true;
+        ready = vs;
         CK(cudaMemcpyAsync(&g->hscr[0], g->mwork, sizeof(u64), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
         work = g->hscr[0];
@@ -1250,8 +1262,7 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                            (const int*)g->dcnt + C_HUB + r, (int*)g->dcnt + C_HUB + r + 1,
                            g->dmap + r, tag_base | (u32)r));
         }
-        hub_pending = phase == 1 && member_ok && r >= 1 && !dense && brnd == 0 &&
-                      chain.len < MST_CHAIN_MAX;
+        hub_pending = phase == 1 && member_ok && r >= 1 && !dense && chain.len < MST_CHAIN_MAX;
         if (hub_pending) {  // (the member-scan decision below first asks whether it can pay)
             Prof p(g, s, MST_K_COMPOSE, r, 2);
             CK(launch_hub_chain(s, (u32)n, chain, Mr, g->hubs, g->dmap + HHUB + r, tag_base | (u32)r));
@@ -1283,8 +1294,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         const bool hy = hy_env ? atoi(hy_env) != 0 : false;
         u32 hub_comps = 0;
         if (hub_pending && !was_v) CKS(wait_word(g, s, HHUB + r, tag_base | (u32)r, &hub_comps));
-        if (phase == 1 && member_ok && r >= 1 && !was_v && !dense && brnd == 0 && hub_pending &&
-            (hy || hub_comps <= 1) &&
+        if (phase == 1 && member_ok && r >= 1 && !was_v && !dense && hub_pending &&
+            ((hy && brnd == 0) || hub_comps <= 1) &&
             nn > 1 && (u64)(nr - nn) * 4 < 3 * nr && moff + nr + 3ull * nn <= 3 * n) {
             // light phase: once the components outside the top hubs' own few record ends, the
             // member scan gives them their exact minima: next to a light pass while the hubs
@@ -1294,7 +1305,11 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             CKS(member_work(r, Mr, true, phi_ready, member_w, member_nbig));
             const bool cheap = member_cheap(member_w);
             member_next = cheap && member_nbig <= 1;
-            hybrid_next = hy && cheap && member_nbig > 1;
+            hybrid_next = hy && brnd == 0 && cheap && member_nbig > 1;
+            if (member_next && brnd != 0) {  // the vertex map becomes Ψ (records: arcs0 next)
+                std::swap(g->phi, g->phi2);
+                phi_ready = true;
+            }
             static const bool dbg1 = getenv("MST_DEBUG_MEMBER") != nullptr;
             if (dbg1) fprintf(stderr, "light round %d: nr %u nn %u member work %llu hub comps %u -> %d %d\n",
                               r, nr, nn, (unsigned long long)member_w, member_nbig, (int)member_next,
@@ -1400,15 +1415,20 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             // one more hook round usually finishes (writing them back cost 0.3 ms)
             // (nor do the light-phase passes: their records are read only a couple more
             // times; measured on RMAT-22 with ~80 % surviving: 49.2 -> 51.1 G edges/s)
+            // light-phase passes (MST_LIGHT_COMPACT): 0 never, 1 adaptive from round 1, 2 always
+            // from round 1, 3 adaptive from round 0
+            static const int lcm = getenv("MST_LIGHT_COMPACT") ? atoi(getenv("MST_LIGHT_COMPACT")) : 0;
+            const bool light_never = phase == 1 && (lcm == 0 || r < (lcm == 3 ? 0 : 1));
             const bool never = g->opt_keep || g->tau == 0 || r == g->st.light_switch_round ||
-                               phase == 1;
+                               light_never;
             int dsh = -1;  // the shard whose pass reports the device-side decision
             for (int j = 0; j < G && dsh < 0; ++j)
                 if (g->shards[j].hi > g->shards[j].lo) dsh = j;
             // (A9 dedup needs the survivors compacted: it always compacts then)
             const bool dedup = g->opt_dedup && g->dd_scratch && G == 1 && !dist && !to_dense &&
                                !never && !member && phase != 1;
-            const bool adaptive = !to_dense && !never && g->tau < 1000 && dsh >= 0 && !dedup;
+            const bool adaptive = !to_dense && !never && g->tau < 1000 && dsh >= 0 && !dedup &&
+                                  !(phase == 1 && lcm == 2);
             const uint4* outbuf = (cur == g->abuf[0]) ? g->abuf[1] : g->abuf[0];
             CompactCtl cc;
             cc.surv = g->dcnt + C_SURV + r;

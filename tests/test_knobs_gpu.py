@@ -40,6 +40,10 @@ KNOBS = [
     {"MST_LIGHT_ONLY0": "1"},
     {"MST_LIGHT_ONLY0": "0"},
     {"MST_MEMBER_SCAN": "0"},    # always a pass over every record after the light phase
+    {"MST_LIGHT_COMPACT": "1"},  # light-phase passes compact (adaptive) from round 1
+    {"MST_LIGHT_COMPACT": "2"},  # ... always from round 1 (member decisions on compacted records)
+    {"MST_LIGHT_COMPACT": "3"},  # ... adaptive from round 0
+    {"MST_LIGHT_COMPACT": "2", "MST_LIGHT_T": "3"},
     {"MST_ADJ_DEDUP": "0"},      # no adjacent-duplicate filter in compacting passes
     {"MST_ADJ_DEDUP": "1"},      # ... on everywhere (also BFS-ordered graphs)
     {"MST_REORDER": "1"},        # hub-first even where the auto rule picks BFS order
