@@ -58,7 +58,10 @@ cudaError_t launch_owner_degree(cudaStream_t st, int nsm, u32 m, const u32* eu, 
                                 u32* odeg, int hi_owner);
 cudaError_t launch_scatter(cudaStream_t st, int nsm, u32 m, const u32* eu, const u32* ev,
                            const unsigned* w, u32* cursor, uint4* arcs, uint2* euv,
-                           int hi_owner, u32 kfmt, u32 vlo, u32 vhi, u32 wbase);
+                           int hi_owner, u32 kfmt, u32 vlo, u32 vhi, u32 wbase, u32 e0 = 0,
+                           u32* wmax = nullptr);
+// records written in the (w << 32 | eid) format -> the packed format kfmt (host-input builds)
+cudaError_t launch_key_format(cudaStream_t st, int nsm, u64 A, uint4* arcs, u32 kfmt);
 // (only the records of owners in [vlo, vhi), at their CSR position minus wbase)
 // light_out != nullptr (MST_OPT_LIGHT_FIRST): also append the records of weight <= *light_t
 // to light_out; every consumer warp reserves blocks of light_blk records (one atomic each)

@@ -358,8 +358,20 @@ mst_status shard_ranges(mst_graph* g, int G, std::vector<u64>& lo, std::vector<u
     return MST_OK;
 }
 
+// Host-array input streamed into the build (mst_create_host / mst_solve_host): the device
+// arrays src/dst/w of build() are staging buffers filled chunk by chunk on a copy stream; the
+// degree pass runs per endpoint chunk as it lands, the weights travel while the layout and row
+// offsets are built, and the scatter runs per weight chunk — the PCIe transfer hides the build.
+struct HostIn {
+    const int32_t *src, *dst;
+    const uint32_t* w;
+    cudaStream_t cs;
+    u64 chunk;                     // edges per chunk
+    std::vector<cudaEvent_t> evs;  // one per endpoint chunk, then one per weight chunk
+};
+
 mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w, int nshards_sim,
-                 int rank, int nranks, int reorder) {
+                 int rank, int nranks, int reorder, HostIn* hin = nullptr) {
     auto t0 = std::chrono::steady_clock::now();
     const u64 n = g->n, m = g->m;
     // reorder: 0 the caller's numbering, 1 the automatic layout, 2 a one-shot solve's (no BFS
@@ -411,8 +423,31 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     u64* dspan;  // [0] sum of |u - v|, [1] the degree argmax
     CKS(galloc(g, &dspan, 2));
     CK(cudaMemsetAsync(dspan, 0, sizeof(u64), g->cst));
-    CK(launch_degree(g->cst, g->nsm, (u32)n, (u32)m, src, dst, w, g->eu, g->ev, deg,
-                     g->dcnt + C_ERR, g->dcnt + C_WMAX, dspan));
+    u64 nch = 0;  // host input: chunks of both copies
+    if (hin) {
+        nch = (m + hin->chunk - 1) / hin->chunk;
+        for (u64 k = 0; k < nch; ++k) {  // endpoints, chunk by chunk; degree per chunk
+            const u64 off = k * hin->chunk, len = std::min<u64>(hin->chunk, m - off);
+            CK(cudaMemcpyAsync(const_cast<int*>(src) + off, hin->src + off, len * 4,
+                               cudaMemcpyHostToDevice, hin->cs));
+            CK(cudaMemcpyAsync(const_cast<int*>(dst) + off, hin->dst + off, len * 4,
+                               cudaMemcpyHostToDevice, hin->cs));
+            CK(cudaEventRecord(hin->evs[k], hin->cs));
+            CK(cudaStreamWaitEvent(g->cst, hin->evs[k], 0));
+            CK(launch_degree(g->cst, g->nsm, (u32)n, (u32)len, src + off, dst + off, nullptr,
+                             g->eu + off, g->ev + off, deg, g->dcnt + C_ERR, g->dcnt + C_WMAX,
+                             dspan));
+        }
+        for (u64 k = 0; k < nch; ++k) {  // then the weights (the scatter waits per chunk)
+            const u64 off = k * hin->chunk, len = std::min<u64>(hin->chunk, m - off);
+            CK(cudaMemcpyAsync(const_cast<unsigned*>(w) + off, hin->w + off, len * 4,
+                               cudaMemcpyHostToDevice, hin->cs));
+            CK(cudaEventRecord(hin->evs[nch + k], hin->cs));
+        }
+    } else {
+        CK(launch_degree(g->cst, g->nsm, (u32)n, (u32)m, src, dst, w, g->eu, g->ev, deg,
+                         g->dcnt + C_ERR, g->dcnt + C_WMAX, dspan));
+    }
     CK(launch_deg_argmax(g->cst, g->nsm, (u32)n, deg, dspan + 1));
     u64 span = 0, dtop = 0;
     CK(cudaMemcpyAsync(&span, dspan, sizeof(u64), cudaMemcpyDeviceToHost, g->cst));
@@ -423,14 +458,17 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     CK(cudaStreamSynchronize(g->cst));
     if (g->hcnt[0]) return fail(MST_EINVAL, "an endpoint is outside [0, n) (n = %lld)", (long long)n);
     mark("degree (reads inputs)");
-    {   // packed minima keys when weight, edge id and a label fit in 63 bits (every handle:
-        // the keys' order is the (w, eid) order, so the MIN of a distributed run is unchanged);
-        // the records carry their key base, so the format is fixed before they are built
+    // packed minima keys when weight, edge id and a label fit in 63 bits (every handle:
+    // the keys' order is the (w, eid) order, so the MIN of a distributed run is unchanged);
+    // the records carry their key base, so the format is fixed before they are built (host
+    // input: after the scatter, which then writes (w << 32 | eid) and takes the largest weight)
+    auto key_format = [&]() {
         const u32 wb = bits_of(g->hcnt[C_WMAX]), eb = bits_of(m > 0 ? (u64)m - 1 : 0),
                   pb = bits_of(n > 0 ? (u64)n - 1 : 0);
         static const char* pk = getenv("MST_PACKED_KEYS");  // "0": always (w << 32) | eid
         if (pb > 0 && wb + eb + pb <= 63 && !(pk && pk[0] == '0')) g->kfmt = (eb + pb) | (pb << 8);
-    }
+    };
+    if (!hin) key_format();
 
     // owner degrees (each non-loop edge once, owned by one endpoint: owner_of())
     // default: the higher internal id (the lower-degree endpoint) owns the record, so the
@@ -529,8 +567,23 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
     g->A0_local = A_loc;
     CKS(galloc(g, &g->arcs0, A_loc));
     CKS(galloc(g, &g->euv, m));
-    CK(launch_scatter(g->cst, g->nsm, (u32)m, g->eu, g->ev, w, cursor, g->arcs0, g->euv, hi_owner,
-                      g->kfmt, (u32)vlo, (u32)vhi, (u32)wbase));
+    if (hin) {
+        for (u64 k = 0; k < nch; ++k) {
+            const u64 off = k * hin->chunk, len = std::min<u64>(hin->chunk, m - off);
+            CK(cudaStreamWaitEvent(g->cst, hin->evs[nch + k], 0));
+            CK(launch_scatter(g->cst, g->nsm, (u32)len, g->eu, g->ev, w, cursor, g->arcs0, g->euv,
+                              hi_owner, 0u, (u32)vlo, (u32)vhi, (u32)wbase, (u32)off,
+                              g->dcnt + C_WMAX));
+        }
+        CK(cudaMemcpyAsync(g->hcnt + C_WMAX, g->dcnt + C_WMAX, sizeof(u32), cudaMemcpyDeviceToHost,
+                           g->cst));
+        CK(cudaStreamSynchronize(g->cst));
+        key_format();
+        CK(launch_key_format(g->cst, g->nsm, A_loc, g->arcs0, g->kfmt));
+    } else {
+        CK(launch_scatter(g->cst, g->nsm, (u32)m, g->eu, g->ev, w, cursor, g->arcs0, g->euv,
+                          hi_owner, g->kfmt, (u32)vlo, (u32)vhi, (u32)wbase));
+    }
     g->vlo = (u32)vlo;
     g->vhi = (u32)vhi;
     g->wbase = (u32)wbase;
@@ -597,7 +650,8 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
 mst_status create_common(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                          const uint32_t* w, int nshards_sim, const uint8_t* id, int rank,
                          int nranks, mst_graph** out, int reorder = 1,
-                         mst_allreduce_min_fn xfn = nullptr, void* xctx = nullptr) {
+                         mst_allreduce_min_fn xfn = nullptr, void* xctx = nullptr,
+                         HostIn* hin = nullptr) {
     if (!out) return fail(MST_EINVAL, "out is NULL");
     *out = nullptr;
     CKS(check_args(n, m, src, dst, w));
@@ -628,7 +682,7 @@ mst_status create_common(int64_t n, int64_t m, const int32_t* src, const int32_t
         release(g);
         return fail(MST_ECUDA, "device synchronisation before the build: %s", cudaGetErrorString(e2));
     }
-    mst_status s = build(g, src, dst, (const unsigned*)w, nshards_sim, rank, nranks, reorder);
+    mst_status s = build(g, src, dst, (const unsigned*)w, nshards_sim, rank, nranks, reorder, hin);
     if (s == MST_OK && id != nullptr) {  // mst_create_dist: NCCL communicator (also 1 rank)
         ncclUniqueId uid;
         memcpy(&uid, id, sizeof uid);
@@ -1707,21 +1761,41 @@ static mst_status create_host_impl(int64_t n, int64_t m, const int32_t* src, con
     cudaError_t e = cudaMallocAsync(&ds, b, st);
     if (e == cudaSuccess) e = cudaMallocAsync(&dd, b, st);
     if (e == cudaSuccess) e = cudaMallocAsync(&dw, b, st);
-    if (e == cudaSuccess && m > 0) e = cudaMemcpyAsync(ds, src, (size_t)m * 4, cudaMemcpyHostToDevice, st);
-    if (e == cudaSuccess && m > 0) e = cudaMemcpyAsync(dd, dst, (size_t)m * 4, cudaMemcpyHostToDevice, st);
-    if (e == cudaSuccess && m > 0) e = cudaMemcpyAsync(dw, w, (size_t)m * 4, cudaMemcpyHostToDevice, st);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);  // (the staging exists before the build)
+    // streamed build (HostIn): the copies overlap the degree pass, layout and scatter;
+    // MST_HOST_STREAM=0: copy everything first, then build
+    static const char* hsv = getenv("MST_HOST_STREAM");
+    const bool stream_in = !(hsv && hsv[0] == '0') && m > 0;
+    // (MST_HOST_CHUNK: edges per chunk, read per call — tests cover many small chunks)
+    const char* hcv = getenv("MST_HOST_CHUNK");
+    const u64 hchunk = hcv && atoll(hcv) > 0 ? (u64)atoll(hcv) : (u64)8 << 20;
+    HostIn hin{src, dst, w, st, hchunk, {}};
+    if (e == cudaSuccess && stream_in) {
+        const u64 nch = ((u64)m + hin.chunk - 1) / hin.chunk;
+        for (u64 k = 0; k < 2 * nch && e == cudaSuccess; ++k) {
+            cudaEvent_t ev;
+            e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+            if (e == cudaSuccess) hin.evs.push_back(ev);
+        }
+    } else if (e == cudaSuccess && m > 0) {
+        e = cudaMemcpyAsync(ds, src, (size_t)m * 4, cudaMemcpyHostToDevice, st);
+        if (e == cudaSuccess) e = cudaMemcpyAsync(dd, dst, (size_t)m * 4, cudaMemcpyHostToDevice, st);
+        if (e == cudaSuccess) e = cudaMemcpyAsync(dw, w, (size_t)m * 4, cudaMemcpyHostToDevice, st);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    }
     mst_status s = MST_OK;
     if (e != cudaSuccess)
         s = fail(e == cudaErrorMemoryAllocation ? MST_ENOMEM : MST_ECUDA, "host->device input copy: %s",
                  cudaGetErrorString(e));
     else
         s = create_common(n, m, (const int32_t*)ds, (const int32_t*)dd, (const uint32_t*)dw, 1,
-                          nullptr, 0, 1, out, reorder);
+                          nullptr, 0, 1, out, reorder, nullptr, nullptr, stream_in ? &hin : nullptr);
+    cudaStreamSynchronize(st);  // (copies still queued after a failed build finish first)
     if (ds) cudaFreeAsync(ds, st);
     if (dd) cudaFreeAsync(dd, st);
     if (dw) cudaFreeAsync(dw, st);
     cudaStreamSynchronize(st);
+    for (cudaEvent_t ev : hin.evs) cudaEventDestroy(ev);
     cudaStreamDestroy(st);
     return s;
 }

@@ -213,6 +213,44 @@ def test_host_paths(lib, oracle_mod, gg):
         assert np.array_equal(ids, o_ids) and tot == o_tot
 
 
+@pytest.mark.parametrize("k,sd", [(4, 0), (3, 0), (2, 2), (5, 4), (1, 0)])
+@pytest.mark.parametrize("chunk", [None, "100003"])
+def test_host_streamed_build(lib, oracle_mod, gg, k, sd, chunk, monkeypatch):
+    """Host-array input: the copies are streamed chunk by chunk under the build (degree per
+    endpoint chunk, scatter per weight chunk, key format fixed afterwards) — bit-exact at full
+    size, with the default chunks and with many small ragged ones (MST_HOST_CHUNK)."""
+    if chunk:
+        monkeypatch.setenv("MST_HOST_CHUNK", chunk)
+    g = gg.config(k, scale_down=sd)
+    o_ids, o_tot = oracle_mod.kruskal(g.n, g.src, g.dst, g.w)
+    pin = lambda a: torch.from_numpy(np.ascontiguousarray(a).view(np.int32)).pin_memory().numpy()  # noqa: E731
+    ps, pd, pw = pin(g.src), pin(g.dst), pin(g.w).view(np.uint32)
+    ids, cnt, tot = lib.mst_solve_host(g.n, ps, pd, pw)
+    assert cnt == len(o_ids) and tot == o_tot and np.array_equal(ids, o_ids)
+    with lib.MSTGraph(g.n, ps, pd, pw, host=True) as h:
+        for _ in range(2):
+            ids, cnt, tot = h.run_host()
+            assert cnt == len(o_ids) and tot == o_tot and np.array_equal(ids, o_ids)
+
+
+def test_host_streamed_errors(lib, oracle_mod, monkeypatch):
+    """An out-of-range endpoint in a later chunk fails the streamed build cleanly (EINVAL),
+    with weight copies still in flight; the library stays usable."""
+    monkeypatch.setenv("MST_HOST_CHUNK", "1000")
+    m = 5000
+    src = np.arange(m, dtype=np.int32) % 100
+    dst = (np.arange(m, dtype=np.int32) * 7 + 1) % 100
+    dst[4321] = 100  # n = 100: out of range, in the fifth chunk
+    with pytest.raises(lib.MSTError) as e:
+        lib.mst_solve_host(100, src, dst, np.ones(m, np.uint32))
+    assert e.value.status == 1
+    dst[4321] = 5
+    w = (np.arange(m, dtype=np.uint32) * 2654435761 % 1000).astype(np.uint32)
+    ids, cnt, tot = lib.mst_solve_host(100, src, dst, w)
+    o_ids, o_tot = oracle_mod.kruskal(100, src, dst, w)
+    assert cnt == len(o_ids) and tot == o_tot and np.array_equal(ids, o_ids)
+
+
 def test_errors(lib):
     with pytest.raises(lib.MSTError) as e:
         lib.MSTGraph(3, dev([0, 1]), dev([1, 3]), dev([1, 1]))
