@@ -96,9 +96,19 @@ cudaError_t launch_hook(cudaStream_t st, u32 nr, const u64* best, u64* best_next
 // tcnt: 2 * hook_tiles(n) words (tile counts, then their exclusive scan)
 // rounds with few hook tiles: the jump also does k_hook_scan's work (n_{r+1} to *nn and to
 // the tagged word hmap, which launch_hook then does not launch)
+// The hub set of launch_hub_chain, computed by the jump's last CTA instead of a launch of its
+// own (on = 0: none); done: a device counter left at 0
+struct HubTask {
+    MapChain chain;
+    int* hubs;
+    u64* hword;
+    u32 tag, n;
+    u32* done;
+    int on;
+};
 cudaError_t launch_jump(cudaStream_t st, int nsm, u32 nr, u32* P, const int* Mtmp, const u32* tcnt,
                         int* Mr, u32* nn, u64* best_next, const int* hub, int* hub_next,
-                        u64* hmap, u32 tag);
+                        u64* hmap, u32 tag, const HubTask* ht = nullptr);
 u64 hook_tiles(u64 n);
 cudaError_t launch_filter_min(cudaStream_t st, int nsm, const u32* a_in, u64 a_max,
                               const uint4* in, const int* M, uint4* out, u64* best, u32 nb,

@@ -93,7 +93,8 @@ constexpr int C_WMAX = C_LT + 1;                   // largest weight (build)
 constexpr int C_TAILN = C_WMAX + 1;                // light-phase tail: labels after it
 constexpr u32 LBLK_MIN = 32, LBLK_MAX = 256;      // light write: records per warp reservation
 constexpr int C_UFU = C_TAILN + 1;                 // union-find variant: unions per round
-constexpr int DCNT_WORDS = C_UFU + MST_MAX_ROUNDS;
+constexpr int C_JDONE = C_UFU + MST_MAX_ROUNDS;    // jump CTAs done (hub set: the last one)
+constexpr int DCNT_WORDS = C_JDONE + 1;
 constexpr int HSURV = MST_MAX_ROUNDS + 1;  // mapped words: [0, HSURV) sizes, [HSURV, 2 HSURV) decisions,
 constexpr int HHUB = 2 * HSURV;            // [2 HSURV, 3 HSURV) the hub sets' component counts
 
@@ -1309,17 +1310,17 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                                                                   // minima cover every edge)
                            dense ? 0u : g->kfmt));  // dense rounds: matrix keys (w << 32 | eid)
         }
+        // (the member-scan decision below first asks whether it can pay: the hub set, computed
+        // by the jump's last CTA)
+        hub_pending = phase == 1 && member_ok && r >= 1 && !dense && chain.len < MST_CHAIN_MAX;
         {   // the jump does not need the host: it reads n_{r+1} on the device and runs
             // while the counts travel to the host
             Prof p(g, s, MST_K_JUMP, r);
+            HubTask ht{chain, g->hubs, g->dmap + HHUB + r, tag_base | (u32)r, (u32)n,
+                       g->dcnt + C_JDONE, hub_pending ? 1 : 0};
             CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, g->tcnt, Mr, g->dcnt + C_NNEXT, bnxt,
                            (const int*)g->dcnt + C_HUB + r, (int*)g->dcnt + C_HUB + r + 1,
-                           g->dmap + r, tag_base | (u32)r));
-        }
-        hub_pending = phase == 1 && member_ok && r >= 1 && !dense && chain.len < MST_CHAIN_MAX;
-        if (hub_pending) {  // (the member-scan decision below first asks whether it can pay)
-            Prof p(g, s, MST_K_COMPOSE, r, 2);
-            CK(launch_hub_chain(s, (u32)n, chain, Mr, g->hubs, g->dmap + HHUB + r, tag_base | (u32)r));
+                           g->dmap + r, tag_base | (u32)r, &ht));
         }
         // one host round trip per round: n_{r+1} (sizes round r's filter),
         // read zero-copy from the word the hook's last tile writes to mapped host memory
