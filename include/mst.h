@@ -129,7 +129,7 @@ enum {
     MST_K_OUTPUT = 5,  /* A11 output compaction                                       */
     MST_K_COMM = 6,    /* A3 cross-GPU MIN (distributed handles)                      */
     MST_K_DENSE = 7,   /* A9 dense rounds over the component min-matrix              */
-    MST_K_LIGHT = 8,   /* A2 light-edge threshold select (sampled radix select)       */
+    MST_K_LIGHT = 8,   /* (unused: the light threshold is selected inside MST_K_INIT)  */
     MST_K_COMPOSE = 9, /* A7 label-map composition (+ the round-0 survival sample)    */
     MST_K_SMALL = 10,  /* A1-A11 in one CTA (MST_OPT_SMALL: graphs that fit smem)      */
     MST_K_DEDUP = 11,  /* A9 sort-based duplicate collapse (MST_OPT_DEDUP)            */

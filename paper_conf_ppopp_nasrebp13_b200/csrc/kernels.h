@@ -81,12 +81,18 @@ u32 pass_warps(int nsm);  // consumer warps of one pass launch, rounded up (the 
 unsigned long long kernel_launches();  // kernels launched by this process so far
 // A1: best = inf (n), msf = 0 (nwords), acc = 0 (nacc), ctr = 0 (nctr), *zero1 = 0,
 // ctr2 = 0 (nctr2: every per-shard, per-round record count of the run)
+// The light-edge threshold selection (launch_light_threshold) done by the init launch's last
+// CTA (on = 0: none)
+struct LightSel {
+    const uint4* arcs;
+    u64 A, target;
+    u32* t_out;
+    u32 s1;
+    int on;
+};
 cudaError_t launch_init(cudaStream_t st, int nsm, u32 n, u64* best, u32 nwords, u32* msf,
-                        u64* acc, u32 nacc, u32* ctr, u32 nctr, u32* zero1, u32* ctr2, u32 nctr2);
-// weight threshold t of the light-edge phase: about `target` of the A records have w <= t
-// (binary search on a 4096-record sample); writes *t
-cudaError_t launch_light_threshold(cudaStream_t st, const uint4* arcs, u64 A, u64 target, u32* t,
-                                   u32 kfmt);
+                        u64* acc, u32 nacc, u32* ctr, u32 nctr, u32* zero1, u32* ctr2, u32 nctr2,
+                        const struct LightSel* ls = nullptr);
 // phi[x] = chain.m[len-1][...chain.m[0][x]] for x < n (-1 stays -1)
 cudaError_t launch_chain_compose(cudaStream_t st, int nsm, u32 n, const MapChain& chain, int* phi);
 // defer (light-edge phase): a component with no (light) edge left is kept, not finished
@@ -96,8 +102,9 @@ cudaError_t launch_hook(cudaStream_t st, u32 nr, const u64* best, u64* best_next
 // tcnt: 2 * hook_tiles(n) words (tile counts, then their exclusive scan)
 // rounds with few hook tiles: the jump also does k_hook_scan's work (n_{r+1} to *nn and to
 // the tagged word hmap, which launch_hook then does not launch)
-// The hub set of launch_hub_chain, computed by the jump's last CTA instead of a launch of its
-// own (on = 0: none); done: a device counter left at 0
+// The hub set of a member-scan decision (the components of internal vertices 0..31 from vertex
+// ids through chain and M_r, sorted, + their distinct live count, also to the tagged mapped
+// word hword), computed by the jump's last CTA (on = 0: none); done: a counter left at 0
 struct HubTask {
     MapChain chain;
     int* hubs;
@@ -171,10 +178,6 @@ cudaError_t launch_compose(cudaStream_t st, int nsm, u32 nb, const int* src, con
 // the hub set's components (the member-scan decision); hubs: 33 ints written first (the
 // sorted labels of the components of vertices 0..31 after Mr, then their number of distinct
 // live labels)
-// the hub set alone, from vertex ids through chain and Mr; its distinct-label count also to the
-// tagged mapped word hword ((tag << 32) | count)
-cudaError_t launch_hub_chain(cudaStream_t st, u32 n, const MapChain& chain, const int* Mr,
-                             int* hubs, u64* hword, u32 tag);
 cudaError_t launch_compose_work(cudaStream_t st, int nsm, u32 nb, const int* src, const int* Mr,
                                 int* phi, int* hubs, const u32* row, const u32* rrow,
                                 u32 vlo, u32 vhi, u64* work);

@@ -1012,18 +1012,6 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     if (g->opt_uf) return run_uf(g, s, out_ids, out_num, out_total, kl0);
     if (small_ok(g)) return run_small(g, s, out_ids, out_num, out_total, kl0);
     const int G = (int)g->shards.size();
-    // ---- A1 init
-    {
-        Prof p(g, s, MST_K_INIT, 0);
-        // best_0 = inf, forest bits, accumulators, per-pass counters (C_SEEN, C_SURV), the
-        // hub label (round 0: vertex 0 itself) and every shard's per-round record counts (a
-        // pass that meets no record must not read a count an earlier run left, ADVICE r1)
-        static_assert(C_SURV == C_SEEN + MST_MAX_ROUNDS, "counter layout");
-        CK(launch_init(s, g->nsm, (u32)n, g->bestA, (u32)std::max<u64>(g->nwords, 1), g->msf,
-                       g->acc, 2 * ACC_SLOTS, g->dcnt + C_SEEN, 2 * MST_MAX_ROUNDS,
-                       g->dcnt + C_HUB, g->dcnt + C_AREC, (u32)G * AREC_STRIDE));
-        if (g->sim) CK(cudaMemsetAsync(g->shard_best, 0xff, n * G * sizeof(u64), s));
-    }
     // light-edge phase (MST_OPT_LIGHT_FIRST): single handle, enough records to pay
     static const u32 lk_env = getenv("MST_LIGHT_K") ? (u32)atoi(getenv("MST_LIGHT_K")) : 0xffffffffu;
     // auto: the light subgraph of a dense near-regular graph must be connected to finish
@@ -1053,34 +1041,47 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     const bool singletons = light_only0 && member_ok;
     g->st.light_switch_round = -1;
     g->st.light_t = 0xffffffffu;
+    // the light threshold t: selected by the init launch's last CTA (no launch of its own)
+    LightSel lsel{};
+    static const char* tf = getenv("MST_LIGHT_T");  // ablation: a fixed threshold
+    if (phase && !tf && g->A0_local > 0) {
+        // auto K = 2 aims a little above 2 n: below t ~ 119 RMAT-22 leaves a small part
+        // uncontracted after the all-records pass (one more full pass: 52.7 -> 44.4 G
+        // edges/s) while t 120-150 is flat; the 4096-record sample puts t within ~+-5
+        // (dense regime, K = 8: aimed at 10 n so that t <= 2 — light degree ~8, a few
+        // vertices without a light edge and one more all-records pass — stays unlikely)
+        // (with member-scan rounds, fewer light records pay: the components the light
+        // phase leaves are finished by member scans, not by a pass over every record;
+        // measured on RMAT-22: t 139 -> 60, 62.8 -> 66.1 G edges/s; t 40: 64.9; with the
+        // light-only round 0: t 60 / 50 / 40 -> 69.2 / 70.8 / 69.1)
+        const bool auto_k = lk_env == 0xffffffffu && g->light_k < 0;
+        const u64 target = !auto_k ? (u64)lk * n : dense_regime ? (u64)10 * n
+                         : member_ok ? (u64)n * 85 / 100 : (u64)23 * n / 10;
+        // a rank samples its own records, aimed at the same fraction of them; every rank
+        // must use the SAME t (a mixed threshold is not a prefix of the (w, id) order),
+        // so the ranks agree on the smallest sampled t
+        const u64 Al = g->A0_local;
+        lsel = LightSel{g->arcs0, Al, (u64)((double)target * Al / g->A0), g->dcnt + C_LT,
+                        (g->kfmt >> 8) ? (g->kfmt & 0xffu) : 32u, 1};
+    }
+    // ---- A1 init
+    {
+        Prof p(g, s, MST_K_INIT, 0);
+        // best_0 = inf, forest bits, accumulators, per-pass counters (C_SEEN, C_SURV), the
+        // hub label (round 0: vertex 0 itself) and every shard's per-round record counts (a
+        // pass that meets no record must not read a count an earlier run left, ADVICE r1)
+        static_assert(C_SURV == C_SEEN + MST_MAX_ROUNDS, "counter layout");
+        CK(launch_init(s, g->nsm, (u32)n, g->bestA, (u32)std::max<u64>(g->nwords, 1), g->msf,
+                       g->acc, 2 * ACC_SLOTS, g->dcnt + C_SEEN, 2 * MST_MAX_ROUNDS,
+                       g->dcnt + C_HUB, g->dcnt + C_AREC, (u32)G * AREC_STRIDE, &lsel));
+        if (g->sim) CK(cudaMemsetAsync(g->shard_best, 0xff, n * G * sizeof(u64), s));
+    }
     if (phase) {
-        Prof p(g, s, MST_K_LIGHT, 0);
-        static const char* tf = getenv("MST_LIGHT_T");  // ablation: a fixed threshold
         if (tf) {
             g->hcnt[C_LT] = (u32)strtoul(tf, nullptr, 10);
             CK(cudaMemcpyAsync(g->dcnt + C_LT, g->hcnt + C_LT, sizeof(u32), cudaMemcpyHostToDevice, s));
-        } else {
-            // auto K = 2 aims a little above 2 n: below t ~ 119 RMAT-22 leaves a small part
-            // uncontracted after the all-records pass (one more full pass: 52.7 -> 44.4 G
-            // edges/s) while t 120-150 is flat; the 4096-record sample puts t within ~+-5
-            // (dense regime, K = 8: aimed at 10 n so that t <= 2 — light degree ~8, a few
-            // vertices without a light edge and one more all-records pass — stays unlikely)
-            // (with member-scan rounds, fewer light records pay: the components the light
-            // phase leaves are finished by member scans, not by a pass over every record;
-            // measured on RMAT-22: t 139 -> 60, 62.8 -> 66.1 G edges/s; t 40: 64.9; with the
-            // light-only round 0: t 60 / 50 / 40 -> 69.2 / 70.8 / 69.1)
-            const bool auto_k = lk_env == 0xffffffffu && g->light_k < 0;
-            const u64 target = !auto_k ? (u64)lk * n : dense_regime ? (u64)10 * n
-                             : member_ok ? (u64)n * 85 / 100 : (u64)23 * n / 10;
-            // a rank samples its own records, aimed at the same fraction of them; every rank
-            // must use the SAME t (a mixed threshold is not a prefix of the (w, id) order),
-            // so the ranks agree on the smallest sampled t
-            const u64 Al = g->A0_local;
-            if (Al == 0)
-                CK(cudaMemsetAsync(g->dcnt + C_LT, 0xff, sizeof(u32), s));
-            else
-                CK(launch_light_threshold(s, g->arcs0, Al, (u64)((double)target * Al / g->A0),
-                                          g->dcnt + C_LT, g->kfmt));
+        } else if (g->A0_local == 0) {
+            CK(cudaMemsetAsync(g->dcnt + C_LT, 0xff, sizeof(u32), s));
         }
         if (dist) {
             Prof p(g, s, MST_K_COMM, 0);
@@ -1228,6 +1229,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
     // worth it below ~1/16 of the streamed bytes)
     auto member_cheap = [&](u64 work) { return work * 16 < 2 * g->A0 / (u64)std::max(1, g->nranks); };
     bool member_next = false;  // the phase-1 check chose a member-scan round for this round
+    int last_member_r = -2;    // the last member-scan round and its work (an upper bound after)
+    u64 last_member_w = 0;
     bool hybrid_next = false;  // ... a hybrid round: light pass + member scan of the small ones
     bool hub_pending = false;  // the jump's hub set count is on its way to the host
     u64 member_w = 0;
@@ -1413,6 +1416,18 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             if (member_next) {
                 member = true;  // (decided by the phase-1 check of this round)
             } else if (phase == 2 && member_ok && cur == g->arcs0 && brnd == 0 &&
+                       (phi_ready || brnd < r) && last_member_r == r - 1) {
+                // right after a member round: the vertices outside the hub's component only
+                // ever join it, so the work cannot have grown — no count, no host round trip
+                if (!phi_ready) {
+                    Prof p(g, s, MST_K_COMPOSE, r);
+                    CK(launch_compose(s, g->nsm, (u32)n, brnd == r - 1 ? chain.m[chain.len - 1] : g->phi,
+                                      Mr, g->phi));
+                    phi_ready = true;
+                }
+                member = true;
+                mwork = last_member_w;
+            } else if (phase == 2 && member_ok && cur == g->arcs0 && brnd == 0 &&
                        (phi_ready || brnd < r)) {
                 u32 nbig = 1;
                 CKS(member_work(r, Mr, false, phi_ready, mwork, nbig));
@@ -1525,6 +1540,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
                 }
                 g->st.member_ends[r] = (int64_t)mwork;
                 g->st.member_round[r] = 1;
+                last_member_r = r;
+                last_member_w = mwork;
             }
             for (int j = 0; j < G && !member; ++j) {
                 Shard& sh = g->shards[j];

@@ -13,8 +13,8 @@ for p in sys.argv[1:]:
           f"frac {d['roofline']['frac'] or 0:.3f} ({d['roofline']['kernel']})  {d['parity']}  "
           f"clk {d['clocks']['sm_mhz']} {d['clocks']['reasons']}  launches {d['gpu_launches']}")
     for k, v in d.get("launch_kinds", {}).items():
-        print(f"   {k:24s} {v['launches_per_step']:5.1f} x {v['avg_launch_ms']*1e3:8.1f} us = "
-              f"{v['ms_per_step']*1e3:8.1f} us/step  frac {v['frac'] or 0:.3f}")
+        print(f"   {k:24s} {v['launches_per_step']:5.1f} x {(v['avg_launch_ms'] or 0)*1e3:8.1f} us = "
+              f"{(v['ms_per_step'] or 0)*1e3:8.1f} us/step  frac {v['frac'] or 0:.3f}")
     for r in d.get("rounds", []):
         print(f"   r{r['r']} {r['kind']:9s} n={r['n_r']:>9} A={r['A_r']:>10} comp={r['compacted']} "
               f"{r['filter_ms']*1e3:7.1f} us frac {r['frac'] or 0:.3f}  hook {r.get('hook_ms', 0)*1e3:6.1f} "
