@@ -71,11 +71,16 @@ typedef struct mst_graph mst_graph; /* opaque; owned by the library */
 mst_status mst_create(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                       const uint32_t* w, mst_graph** out);
 
-/* mst_create_host — as mst_create but src/dst/w are HOST pointers (pageable or pinned).
- * The arrays are copied to stream-ordered device buffers first (copy engines; pinned arrays
- * reach the bus rate, ~55 GB/s, pageable ones are staged by the driver), then built as by
- * mst_create (input transferred to the GPU). The build's small pinned host
- * buffers come from a process-wide free list (no page-locking per handle). */
+/* mst_create_host — as mst_create but src/dst/w are HOST pointers (pageable or pinned),
+ * read only during the call. The arrays are streamed to stream-ordered device buffers in
+ * 8 M-edge chunks (copy engines; pinned arrays reach the bus rate, ~55 GB/s, pageable ones
+ * are staged by the driver) WHILE the build consumes them: the degree/validation pass runs
+ * per endpoint chunk, the layout while the weights travel, the record scatter per weight
+ * chunk (input transferred to the GPU) — the result is the same handle as
+ * mst_create's. An endpoint outside [0, n) in any chunk: MST_EINVAL, nothing leaked.
+ * (MST_HOST_STREAM=0 copies everything first; MST_HOST_CHUNK sets the chunk, in edges.)
+ * The build's small pinned host buffers come from a process-wide free list (no
+ * page-locking per handle). */
 mst_status mst_create_host(int64_t n, int64_t m, const int32_t* src, const int32_t* dst,
                            const uint32_t* w, mst_graph** out);
 

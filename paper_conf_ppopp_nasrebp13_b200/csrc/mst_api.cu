@@ -1305,22 +1305,24 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             vround = false;
             nn = v_nn;
         } else {
-        {
-            Prof p(g, s, MST_K_HOOK, r);
-            CK(launch_hook(s, nr, bcur, bnxt, g->dmap + r, tag_base | (u32)r, g->euv, chain, g->P,
-                           g->Mtmp, g->msf, g->acc, g->tcnt, g->dcnt + C_NNEXT,
-                           phase == 1 && (r > 0 || (light_only0 && !singletons)),  // (else round 0's
-                                                                  // minima cover every edge)
-                           dense ? 0u : g->kfmt));  // dense rounds: matrix keys (w << 32 | eid)
-        }
         // (the member-scan decision below first asks whether it can pay: the hub set, computed
         // by the jump's last CTA)
         hub_pending = phase == 1 && member_ok && r >= 1 && !dense && chain.len < MST_CHAIN_MAX;
-        {   // the jump does not need the host: it reads n_{r+1} on the device and runs
-            // while the counts travel to the host
+        const bool hdefer = phase == 1 && (r > 0 || (light_only0 && !singletons));  // (else
+                                                  // round 0's minima cover every edge)
+        const u32 hkfmt = dense ? 0u : g->kfmt;  // dense rounds: matrix keys (w << 32 | eid)
+        HubTask ht{chain, g->hubs, g->dmap + HHUB + r, tag_base | (u32)r, (u32)n,
+                   g->dcnt + C_JDONE, hub_pending ? 1 : 0};
+        {
+            {
+                Prof p(g, s, MST_K_HOOK, r);
+                CK(launch_hook(s, nr, bcur, bnxt, g->dmap + r, tag_base | (u32)r, g->euv, chain,
+                               g->P, g->Mtmp, g->msf, g->acc, g->tcnt, g->dcnt + C_NNEXT, hdefer,
+                               hkfmt));
+            }
+            // the jump does not need the host: it reads n_{r+1} on the device and runs while
+            // the counts travel to the host
             Prof p(g, s, MST_K_JUMP, r);
-            HubTask ht{chain, g->hubs, g->dmap + HHUB + r, tag_base | (u32)r, (u32)n,
-                       g->dcnt + C_JDONE, hub_pending ? 1 : 0};
             CK(launch_jump(s, g->nsm, nr, g->P, g->Mtmp, g->tcnt, Mr, g->dcnt + C_NNEXT, bnxt,
                            (const int*)g->dcnt + C_HUB + r, (int*)g->dcnt + C_HUB + r + 1,
                            g->dmap + r, tag_base | (u32)r, &ht));

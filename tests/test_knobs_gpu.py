@@ -44,6 +44,8 @@ KNOBS = [
     {"MST_LIGHT_COMPACT": "2"},  # ... always from round 1 (member decisions on compacted records)
     {"MST_LIGHT_COMPACT": "3"},  # ... adaptive from round 0
     {"MST_LIGHT_COMPACT": "2", "MST_LIGHT_T": "3"},
+    {"MST_TX_DEDUP": "0"},       # dense transition: no warp merge of equal cells
+    {"MST_TX_DEDUP": "1"},       # ... also without a hub row
     {"MST_ADJ_DEDUP": "0"},      # no adjacent-duplicate filter in compacting passes
     {"MST_ADJ_DEDUP": "1"},      # ... on everywhere (also BFS-ordered graphs)
     {"MST_REORDER": "1"},        # hub-first even where the auto rule picks BFS order
