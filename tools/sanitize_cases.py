@@ -3,7 +3,9 @@ graphs small enough for memcheck/racecheck/synccheck, each checked against the o
 
 grid64 through the multi-kernel path (device tail on and off, light phase forced, keep-edges,
 union-find, sharded simulation) and through the one-CTA path; small random multigraphs with
-ties, loops and parallel edges; a scaled RMAT with the dense transition and the hub row.
+ties, loops and parallel edges; a scaled RMAT with the dense transition and the hub row (and
+the light phase: threshold select in the init launch, member scans, the jump's hub set); the
+streamed host-input build.
 """
 import os
 import sys
@@ -63,6 +65,16 @@ def main():
     r = graphgen.config(4, s=1, scale_down=9)  # RMAT 8 K vertices, 131 K edges
     check("rmat-sd9", r.n, r.src, r.dst, r.w, base)
     check("rmat-sd9 no-tail", r.n, r.src, r.dst, r.w, base + [(TAIL, 0), (LF, 0)])
+    # streamed host-input build (degree per endpoint chunk, scatter per weight chunk, key format
+    # afterwards), one-shot and persistent, in many small chunks
+    os.environ["MST_HOST_CHUNK"] = "20011"
+    o_ids, o_tot = oracle.kruskal(r.n, r.src, r.dst, r.w)
+    ids, cnt, tot = lib.mst_solve_host(r.n, r.src, r.dst, r.w)
+    assert cnt == len(o_ids) and tot == o_tot and np.array_equal(ids, o_ids), "host solve"
+    with lib.MSTGraph(r.n, r.src, r.dst, r.w, host=True) as h:
+        ids, cnt, tot = h.run_host()
+    assert cnt == len(o_ids) and tot == o_tot and np.array_equal(ids, o_ids), "host handle"
+    print("ok rmat-sd9 host streamed", flush=True)
 
 
 if __name__ == "__main__":
