@@ -15,6 +15,7 @@
 //
 // Nothing is allocated inside mst_run (PAPER.md L259 pre-allocation). All work is enqueued
 // on the caller's stream.
+#include <nvtx3/nvToolsExt.h>
 #include <cuda_runtime.h>
 #include <nccl.h>
 
@@ -290,6 +291,28 @@ cudaEvent_t next_event(mst_graph* g) {
     return g->evpool[g->evused++];
 }
 
+// NVTX ranges: every profiled launch group is also a host range named by its
+// kind with the round as payload (nvtx3 is header-only: without an attached tool a push/pop
+// is a check of one function pointer)
+const char* const kNvtxName[MST_K_COUNT] = {"mst init", "mst min0 (A2)", "mst hook (A4/A6)",
+                                            "mst jump (A5/A6)", "mst filter (A8)", "mst output (A11)",
+                                            "mst comm (A3)", "mst dense (A9)", "mst light",
+                                            "mst compose (A7)", "mst small (A1-A11)", "mst dedup (A9)"};
+void nvtx_push(const char* name, int payload) {
+    nvtxEventAttributes_t ea{};
+    ea.version = NVTX_VERSION;
+    ea.size = NVTX_EVENT_ATTRIB_STRUCT_SIZE;
+    ea.messageType = NVTX_MESSAGE_TYPE_ASCII;
+    ea.message.ascii = name;
+    ea.payloadType = NVTX_PAYLOAD_TYPE_INT32;
+    ea.payload.iValue = payload;
+    nvtxRangePushEx(&ea);
+}
+struct NvtxRange {
+    NvtxRange(const char* name, int payload = 0) { nvtx_push(name, payload); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
+
 struct Prof {
     mst_graph* g;
     cudaStream_t s;
@@ -297,12 +320,14 @@ struct Prof {
     cudaEvent_t a = nullptr;
     Prof(mst_graph* g_, cudaStream_t s_, int kind_, int round_, int sub_ = 0, int shard_ = 0)
         : g(g_), s(s_), kind(kind_), round(round_), sub(sub_), shard(shard_) {
+        nvtx_push(kind >= 0 && kind < MST_K_COUNT ? kNvtxName[kind] : "mst", round);
         if (g->prof) {
             a = next_event(g);
             cudaEventRecord(a, s);
         }
     }
     ~Prof() {
+        nvtxRangePop();
         if (g->prof) {
             cudaEvent_t b = next_event(g);
             cudaEventRecord(b, s);
@@ -683,7 +708,11 @@ mst_status create_common(int64_t n, int64_t m, const int32_t* src, const int32_t
         release(g);
         return fail(MST_ECUDA, "device synchronisation before the build: %s", cudaGetErrorString(e2));
     }
-    mst_status s = build(g, src, dst, (const unsigned*)w, nshards_sim, rank, nranks, reorder, hin);
+    mst_status s;
+    {
+        NvtxRange range("mst_create (A0 build)", (int)std::min<int64_t>(m, INT32_MAX));
+        s = build(g, src, dst, (const unsigned*)w, nshards_sim, rank, nranks, reorder, hin);
+    }
     if (s == MST_OK && id != nullptr) {  // mst_create_dist: NCCL communicator (also 1 rank)
         ncclUniqueId uid;
         memcpy(&uid, id, sizeof uid);
@@ -1834,6 +1863,7 @@ mst_status mst_run(mst_graph* g, mst_stream_t stream, int32_t* out_edge_ids,
         if (g->broken) return fail(MST_EINVAL, "handle is unusable after an earlier error");
         if (!out_num_edges || !out_total_weight) return fail(MST_EINVAL, "null output pointer");
         if (!out_edge_ids && g->n > 1) return fail(MST_EINVAL, "out_edge_ids is NULL");
+        NvtxRange range("mst_run", (int)std::min<int64_t>(g->n, INT32_MAX));
         mst_status s = run_impl(g, (cudaStream_t)stream, out_edge_ids, out_num_edges, out_total_weight);
         if (s != MST_OK) {
             g->broken = true;
