@@ -623,7 +623,9 @@ mst_status build(mst_graph* g, const int* src, const int* dst, const unsigned* w
         CKS(galloc(g, &g->ridx, A_loc));
         CKS(galloc(g, &g->mwork, 1));
         CKS(galloc(g, &g->hubs, 64));
-        CKS(galloc(g, &g->phi2, n));
+        // (the spare vertex map only serves the light-compaction ablation, MST_LIGHT_COMPACT)
+        const char* lcv = getenv("MST_LIGHT_COMPACT");
+        if (lcv && atoi(lcv) != 0) CKS(galloc(g, &g->phi2, n));
         u32* rpc;  // (per-CTA counts of the hot vertices; build time only)
         CKS(galloc(g, &rpc, reverse_index_scratch(g->nsm, (u32)n)));
         CK(launch_reverse_index(g->cst, g->nsm, (u32)n, A_loc, g->arcs0, rdeg, g->rrow, cursor,
@@ -1521,7 +1523,8 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
             // light-phase passes (MST_LIGHT_COMPACT): 0 never, 1 adaptive from round 1, 2 always
             // from round 1, 3 adaptive from round 0
             static const int lcm = getenv("MST_LIGHT_COMPACT") ? atoi(getenv("MST_LIGHT_COMPACT")) : 0;
-            const bool light_never = phase == 1 && (lcm == 0 || r < (lcm == 3 ? 0 : 1));
+            const bool light_never = phase == 1 && (lcm == 0 || r < (lcm == 3 ? 0 : 1) ||
+                                                    (member_ok && !g->phi2));
             const bool never = g->opt_keep || g->tau == 0 || r == g->st.light_switch_round ||
                                light_never;
             int dsh = -1;  // the shard whose pass reports the device-side decision
