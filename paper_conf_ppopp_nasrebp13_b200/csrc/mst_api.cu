@@ -1086,9 +1086,12 @@ mst_status run_impl(mst_graph* g, cudaStream_t s, int32_t* out_ids, int64_t* out
         // measured on RMAT-22: t 139 -> 60, 62.8 -> 66.1 G edges/s; t 40: 64.9; with the
         // light-only round 0: t 60 / 50 / 40 -> 69.2 / 70.8 / 69.1; round 2, session 2, with
         // cheaper light passes, medians of 3: t 20 / 26 / 31 / 36 / 42 / ~54 (0.85 n) ->
-        // 78.5 / 80.6 / 81.1 / 82.2 / 82.3 / 79.3: aimed at 0.62 n, t ~ 39)
+        // 78.5 / 80.6 / 81.1 / 82.2 / 82.3 / 79.3: aimed at 0.62 n, t ~ 39; dense: t = 3 has a
+        // cliff on some seeds (113 vs 216 G edges/s) and t <= 2 everywhere, so its target is
+        // 12 n — t 5 +- 1 from the 4096-record sample — rather than 10 n, where t = 3 came out
+        // of the sample ~8 % of the time)
         const bool auto_k = lk_env == 0xffffffffu && g->light_k < 0;
-        const u64 target = !auto_k ? (u64)lk * n : dense_regime ? (u64)10 * n
+        const u64 target = !auto_k ? (u64)lk * n : dense_regime ? (u64)12 * n
                          : member_ok ? (u64)n * 62 / 100 : (u64)23 * n / 10;
         // a rank samples its own records, aimed at the same fraction of them; every rank
         // must use the SAME t (a mixed threshold is not a prefix of the (w, id) order),
