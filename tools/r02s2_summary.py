@@ -20,7 +20,7 @@ out = ["# Round 2, session 2 — ncu summaries and bench lines on the final code
        "each bench line (`launch_kinds`), not absolute times.", "", sh("python tools/results_table.py profiles r02s2_bench_")]
 notes = {
     "rmat22": """* A2 extraction (first row): ~1,083 MB of DRAM for 1,074 MB of records read + the light records written;
-  ~161 µs cold = 6.7 TB/s of algorithmic bytes; live 0.98 of the measured 6,545 GB/s. The light minima pass (row 2)
+  ~161 µs cold = 6.7 TB/s of algorithmic bytes; live 0.98 of the measured 6,551 GB/s. The light minima pass (row 2)
   and the four light FILTER passes (~3 M records each, 44–48 % L2 hit) are bound by the label gathers into the 16.8 MB
   vertex map, not bytes.
 * Member scans: ~0.5 M record ends of the small components, then a last one over a few hundred.""",

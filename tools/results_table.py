@@ -6,7 +6,7 @@ import os
 import sys
 
 d, pre = sys.argv[1], sys.argv[2]
-print("| Config | Bit-exact | Edges/s (device) | ms/step | Dominant kernel (frac of 6,545 GB/s) | A2 frac | A8 frac | "
+print("| Config | Bit-exact | Edges/s (device) | ms/step | Dominant kernel (frac of the measured HBM peak) | A2 frac | A8 frac | "
       "DRAM / algorithmic bytes | Light phase | e2e edges/s | Oracle (1 core) | GPU launches |")
 print("|---|---|---|---|---|---|---|---|---|---|---|---|")
 for w in ["grid64", "uniform", "road", "rmat22", "dense"]:
